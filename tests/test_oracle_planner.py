@@ -1,0 +1,76 @@
+"""Pins for the oracle GroupBy planner (§5.2).
+
+The plan does not change any depth, so parity is pinned by invariants, by hand-built
+examples worked from Rule 1 / Rule 2 by hand, and by the direction of the paper's
+sharing claim (GroupBy raises SD over random grouping)."""
+from __future__ import annotations
+
+import numpy as np
+
+import ibfs_gen
+import oracle
+from oracle import planner, stats
+
+
+def _csr(nv, pairs):
+    g = oracle.OracleGraph.from_edges(ibfs_gen.from_pairs(nv, pairs))
+    return g.adjacency()
+
+
+def test_two_hub_example_by_hand():
+    # hub A = 0 with leaves 2..9 (deg 8); hub B = 1 with leaves 10..15 (deg 6);
+    # 16 isolated; 17-18 a separate edge (no neighbour above q).
+    pairs = [(0, x) for x in range(2, 10)] + [(1, x) for x in range(10, 16)] + [(17, 18)]
+    off, adj = _csr(19, pairs)
+    sources = np.array([2, 10, 3, 11, 4, 12, 5, 13, 6, 7, 16, 17], dtype=np.uint32)
+    perm = planner.groupby(off, adj, sources, group_bits=4, q=5)
+    # Rule 1 (deg 1 < p=4) and Rule 2 (shared neighbour with deg > q=5) hold for the
+    # leaves; buckets are visited by hub degree (A first); full groups of W=4 first,
+    # then A's leftovers, then the isolated source, then the random remainder.
+    assert perm.tolist() == [0, 2, 4, 6, 1, 3, 5, 7, 8, 9, 10, 11]
+
+
+def test_uniform_graph_fallback_any_degree():
+    # cycle: every degree is 2 <= q, so the hub is the max-degree neighbour of any
+    # degree, ties to the lower id ("share some common vertices").
+    n = 8
+    off, adj = _csr(n, [(i, (i + 1) % n) for i in range(n)])
+    hub, _ = planner.hubs(off, adj, np.arange(n, dtype=np.uint32), q=128)
+    exp = [min((i - 1) % n, (i + 1) % n) for i in range(n)]
+    assert hub.tolist() == exp
+
+
+def test_permutation_invariants_and_determinism():
+    el = ibfs_gen.rmat(12, 16, ibfs_gen.KRONECKER, seed=1)
+    g = oracle.OracleGraph.from_edges(el)
+    off, adj = g.adjacency()
+    src = ibfs_gen.sample_sources(el, 300, seed=2)
+    for W in (32, 64, 128):
+        p1 = planner.groupby(off, adj, src, W)
+        p2 = planner.groupby(off, adj, src, W)
+        assert sorted(p1.tolist()) == list(range(300))
+        np.testing.assert_array_equal(p1, p2)
+    r = planner.random_plan(300, 3)
+    assert sorted(r.tolist()) == list(range(300))
+    assert planner.shuffle([], 1) == [] and planner.shuffle([7], 1) == [7]
+
+
+def test_groupby_raises_sharing_on_apsp_pool():
+    el = ibfs_gen.rmat(12, 16, ibfs_gen.KRONECKER, seed=1)
+    g = oracle.OracleGraph.from_edges(el)
+    off, adj = g.adjacency()
+    deg = np.diff(off)
+    src = np.flatnonzero(deg > 0).astype(np.uint32)
+    W = 64
+    res = g.bfs(src)
+
+    def mean_sd(perm):
+        sds = []
+        for k in range(len(perm) // W):
+            rows = res.depths[perm[k * W:(k + 1) * W]]
+            sds.append(stats.sharing_degree(rows))
+        return float(np.mean(sds))
+
+    sd_g = mean_sd(planner.groupby(off, adj, src, W))
+    sd_r = mean_sd(planner.random_plan(len(src), 3))
+    assert sd_g > 1.2 * sd_r

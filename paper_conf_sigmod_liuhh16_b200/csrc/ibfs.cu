@@ -1,0 +1,865 @@
+// ibfs.cu -- C ABI of libibfs.so (include/ibfs.h): graph loading, the batch/level loop
+// around the sm_100a kernels of kernels.cuh, statistics, allocator hook.
+//
+// Host orchestration of one ibfs_run_ex call:
+//   groups = consecutive chunks of group_bits sources; G groups run per launch batch
+//   (all of a batch's groups share each level launch; each keeps its own direction).
+//   per batch: init_state + init_sources, then per level l = 1, 2, ...:
+//     expand_kernel(l), commit_kernel(l); every LEVELS_PER_CHECK levels the batch's
+//     done-counter is copied to pinned host memory, with one chunk of look-ahead so the
+//     device never waits for the host; kernels of a finished batch exit immediately.
+//   then m_s (+ digest) finalize outside the timed window; D2H of rows if the caller's
+//   buffer is on the host.
+#include <cuda_runtime.h>
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/ibfs.h"
+#include "kernels.cuh"
+#include "plan.h"
+
+using namespace ibfs;
+
+// ------------------------------------------------------------------ error plumbing ----
+namespace {
+thread_local std::string g_last_error;
+
+struct IbfsError {
+  int code;
+  std::string msg;
+};
+
+[[noreturn]] void fail(int code, const std::string &msg) { throw IbfsError{code, msg}; }
+
+void cuda_check(cudaError_t e, const char *what) {
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    int code = (e == cudaErrorMemoryAllocation) ? IBFS_E_NOMEM : IBFS_E_CUDA;
+    fail(code, std::string(what) + ": " + cudaGetErrorString(e));
+  }
+}
+#define CK(x) cuda_check((x), #x)
+
+template <typename F>
+int guarded(F &&f) {
+  try {
+    f();
+    g_last_error.clear();
+    return IBFS_OK;
+  } catch (const IbfsError &e) {
+    g_last_error = e.msg;
+    return e.code;
+  } catch (const std::bad_alloc &) {
+    g_last_error = "host allocation failed";
+    return IBFS_E_NOMEM;
+  } catch (...) {
+    g_last_error = "unknown internal error";
+    return IBFS_E_CUDA;
+  }
+}
+
+// Restores the caller's current device on scope exit.
+struct DeviceScope {
+  int prev = -1;
+  explicit DeviceScope(int dev) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+      cudaGetLastError();
+      fail(IBFS_E_CUDA, "no CUDA device available (libibfs has no CPU fallback)");
+    }
+    if (dev < 0 || dev >= n) fail(IBFS_E_INVALID, "device index out of range");
+    CK(cudaGetDevice(&prev));
+    CK(cudaSetDevice(dev));
+  }
+  ~DeviceScope() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// ------------------------------------------------------------------------ memory ----
+struct Allocator {
+  void *(*alloc)(size_t, int, void *) = nullptr;
+  void (*release)(void *, int, void *) = nullptr;
+  void *ctx = nullptr;
+};
+std::mutex g_alloc_mu;
+Allocator g_alloc;
+
+Allocator current_allocator() {
+  std::lock_guard<std::mutex> lk(g_alloc_mu);
+  return g_alloc;
+}
+
+// Device scratch owned by one call: caller allocator if installed, else the stream-
+// ordered pool (cudaMallocAsync; the pool keeps memory across calls).
+class Scratch {
+ public:
+  Scratch(int dev, cudaStream_t s) : dev_(dev), stream_(s), al_(current_allocator()) {}
+  ~Scratch() {
+    for (void *p : ptrs_) {
+      if (al_.alloc) al_.release(p, dev_, al_.ctx);
+      else cudaFreeAsync(p, stream_);
+    }
+  }
+  template <typename T>
+  T *get(size_t count) {
+    size_t bytes = std::max<size_t>(count * sizeof(T), 256);
+    void *p = nullptr;
+    if (al_.alloc) {
+      p = al_.alloc(bytes, dev_, al_.ctx);
+      if (!p) fail(IBFS_E_NOMEM, "caller allocator returned NULL");
+    } else {
+      cudaError_t e = cudaMallocAsync(&p, bytes, stream_);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(IBFS_E_NOMEM, "cudaMallocAsync(" + std::to_string(bytes) + " bytes) failed");
+      }
+    }
+    ptrs_.push_back(p);
+    return static_cast<T *>(p);
+  }
+
+ private:
+  int dev_;
+  cudaStream_t stream_;
+  Allocator al_;
+  std::vector<void *> ptrs_;
+};
+
+void set_pool_threshold(int dev) {
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  cudaGetLastError();
+}
+
+bool is_device_ptr(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+struct HostPinned {
+  void *p = nullptr;
+  explicit HostPinned(size_t bytes) { CK(cudaMallocHost(&p, bytes)); }
+  ~HostPinned() {
+    if (p) cudaFreeHost(p);
+  }
+};
+
+}  // namespace
+
+// -------------------------------------------------------------------------- graph ----
+struct ibfs_graph {
+  int device = 0;
+  uint32_t nv = 0;
+  uint64_t ne = 0;
+  uint32_t max_deg = 0;
+  uint64_t nv_active = 0;
+  unsigned long long *d_off = nullptr;
+  uint32_t *d_adj = nullptr;
+  uint32_t *d_deg = nullptr;
+  HubChunk *d_chunks = nullptr;
+  uint32_t n_chunks = 0;
+  uint32_t *d_tiles = nullptr;
+  uint32_t n_tiles = 0;
+  std::vector<uint64_t> h_off;  // host copy (tiling, planner)
+  int num_sms = 148;
+  int expand_blocks_per_sm = 1;
+};
+
+namespace {
+
+void graph_release(ibfs_graph *g) {
+  if (!g) return;
+  int prev = -1;
+  if (cudaGetDevice(&prev) == cudaSuccess) cudaSetDevice(g->device);
+  cudaFree(g->d_off);
+  cudaFree(g->d_adj);
+  cudaFree(g->d_deg);
+  cudaFree(g->d_chunks);
+  cudaFree(g->d_tiles);
+  if (prev >= 0) cudaSetDevice(prev);
+  cudaGetLastError();
+  delete g;
+}
+
+__global__ void degree_kernel(const unsigned long long *off, uint32_t nv, uint32_t *deg,
+                              unsigned long long *maxdeg_nz) {
+  uint32_t local_max = 0, local_nz = 0;
+  for (size_t v = (size_t)blockIdx.x * blockDim.x + threadIdx.x; v < nv;
+       v += (size_t)gridDim.x * blockDim.x) {
+    unsigned long long d = off[v + 1] - off[v];
+    uint32_t d32 = d > 0xffffffffull ? 0xffffffffu : (uint32_t)d;
+    deg[v] = d32;
+    local_max = max(local_max, d32);
+    local_nz += d32 > 0;
+  }
+  local_max = __reduce_max_sync(FULL, local_max);
+  local_nz = __reduce_add_sync(FULL, local_nz);
+  if ((threadIdx.x & 31) == 0) {
+    atomicMax(&maxdeg_nz[0], (unsigned long long)local_max);
+    atomicAdd(&maxdeg_nz[1], (unsigned long long)local_nz);
+  }
+}
+
+__global__ void max_id_kernel(const uint32_t *adj, unsigned long long ne, uint32_t *mx) {
+  uint32_t m = 0;
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < ne;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    m = max(m, adj[i]);
+  m = __reduce_max_sync(FULL, m);
+  if ((threadIdx.x & 31) == 0) atomicMax(mx, m);
+}
+
+// Static work decomposition: hub chunks for deg > HUB_T, and tiles of
+// consecutive vertices holding <= V_TILE vertices and <= E_TILE non-hub edges.
+void build_decomposition(ibfs_graph *g) {
+  std::vector<HubChunk> chunks;
+  std::vector<uint32_t> tiles;
+  tiles.push_back(0);
+  uint64_t cur_e = 0;
+  uint32_t cur_n = 0;
+  for (uint32_t v = 0; v < g->nv; ++v) {
+    uint64_t d = g->h_off[v + 1] - g->h_off[v];
+    uint64_t dn = d > (uint64_t)HUB_T ? 0 : d;
+    if (d > (uint64_t)HUB_T) {
+      uint32_t first = 1;
+      for (uint64_t e = g->h_off[v]; e < g->h_off[v + 1]; e += CHUNK) {
+        HubChunk c;
+        c.e0 = e;
+        c.e1 = std::min<uint64_t>(e + CHUNK, g->h_off[v + 1]);
+        c.v = v;
+        c.first = first;
+        first = 0;
+        chunks.push_back(c);
+      }
+    }
+    if (cur_n > 0 && (cur_n == (uint32_t)V_TILE || cur_e + dn > (uint64_t)E_TILE)) {
+      tiles.push_back(v);
+      cur_n = 0;
+      cur_e = 0;
+    }
+    cur_n++;
+    cur_e += dn;
+  }
+  tiles.push_back(g->nv);
+  g->n_tiles = (uint32_t)(tiles.size() - 1);
+  g->n_chunks = (uint32_t)chunks.size();
+  CK(cudaMalloc(&g->d_tiles, tiles.size() * sizeof(uint32_t)));
+  CK(cudaMemcpy(g->d_tiles, tiles.data(), tiles.size() * sizeof(uint32_t), cudaMemcpyHostToDevice));
+  CK(cudaMalloc(&g->d_chunks, std::max<size_t>(chunks.size(), 1) * sizeof(HubChunk)));
+  if (!chunks.empty())
+    CK(cudaMemcpy(g->d_chunks, chunks.data(), chunks.size() * sizeof(HubChunk), cudaMemcpyHostToDevice));
+}
+
+// Degrees, max degree, tiles; offsets must be in g->d_off and g->h_off.
+void finish_graph(ibfs_graph *g) {
+  CK(cudaMalloc(&g->d_deg, std::max<size_t>(g->nv, 1) * sizeof(uint32_t)));
+  unsigned long long *d_stats = nullptr;
+  CK(cudaMalloc(&d_stats, 2 * sizeof(unsigned long long)));
+  CK(cudaMemset(d_stats, 0, 2 * sizeof(unsigned long long)));
+  degree_kernel<<<1024, 256>>>(g->d_off, g->nv, g->d_deg, d_stats);
+  CK(cudaGetLastError());
+  unsigned long long h[2];
+  CK(cudaMemcpy(h, d_stats, sizeof(h), cudaMemcpyDeviceToHost));
+  cudaFree(d_stats);
+  for (uint32_t v = 0; v < g->nv; ++v)
+    if (g->h_off[v + 1] - g->h_off[v] > 0xffffffffull)
+      fail(IBFS_E_UNSUPPORTED, "vertex degree >= 2^32");
+  g->max_deg = (uint32_t)h[0];
+  g->nv_active = h[1];
+  build_decomposition(g);
+  int dev = g->device;
+  CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev));
+  int occ = 1;
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, expand_kernel<u128>, BLOCK, 0));
+  g->expand_blocks_per_sm = std::max(1, occ);
+  set_pool_threshold(dev);
+}
+
+__global__ void explode_kernel(const uint32_t *u, const uint32_t *v, unsigned long long m,
+                               uint32_t *keys, uint32_t *vals, unsigned long long *deg, uint32_t nv,
+                               uint32_t *bad) {
+  for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m;
+       e += (unsigned long long)gridDim.x * blockDim.x) {
+    uint32_t a = u[e], b = v[e];
+    if (a >= nv || b >= nv) {
+      *bad = 1;
+      a = 0;
+      b = 0;
+    }
+    keys[2 * e] = a;
+    vals[2 * e] = b;
+    keys[2 * e + 1] = b;
+    vals[2 * e + 1] = a;
+    atomicAdd(deg + a, 1ull);
+    atomicAdd(deg + b, 1ull);
+  }
+}
+
+}  // namespace
+
+extern "C" int ibfs_version(void) { return 10000; }
+
+extern "C" const char *ibfs_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" int ibfs_load_csr(int device, uint32_t nv, uint64_t ne, const uint64_t *offsets,
+                             const uint32_t *adj, const uint64_t *rev_offsets,
+                             const uint32_t *rev_adj, ibfs_graph **out_graph) {
+  return guarded([&] {
+    if (!out_graph) fail(IBFS_E_INVALID, "out_graph is NULL");
+    *out_graph = nullptr;
+    if (nv == 0) fail(IBFS_E_INVALID, "nv must be >= 1");
+    if (!offsets || (ne > 0 && !adj)) fail(IBFS_E_INVALID, "offsets/adj is NULL");
+    if (ne >= (1ull << 40)) fail(IBFS_E_INVALID, "ne too large");
+    if (rev_offsets || rev_adj)
+      fail(IBFS_E_UNSUPPORTED, "directed graphs (reverse CSR) are not implemented in this build");
+    DeviceScope ds(device);
+    ibfs_graph *g = new ibfs_graph();
+    try {
+      g->device = device;
+      g->nv = nv;
+      g->ne = ne;
+      g->h_off.resize((size_t)nv + 1);
+      CK(cudaMemcpy(g->h_off.data(), offsets, ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyDefault));
+      if (g->h_off[0] != 0 || g->h_off[nv] != ne) fail(IBFS_E_INVALID, "offsets[0] != 0 or offsets[nv] != ne");
+      for (uint32_t v = 0; v < nv; ++v)
+        if (g->h_off[v + 1] < g->h_off[v]) fail(IBFS_E_INVALID, "offsets not non-decreasing");
+      CK(cudaMalloc(&g->d_off, ((size_t)nv + 1) * sizeof(unsigned long long)));
+      CK(cudaMemcpy(g->d_off, g->h_off.data(), ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
+      CK(cudaMalloc(&g->d_adj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
+      if (ne) CK(cudaMemcpy(g->d_adj, adj, ne * sizeof(uint32_t), cudaMemcpyDefault));
+      if (ne) {
+        uint32_t *d_mx = nullptr;
+        CK(cudaMalloc(&d_mx, sizeof(uint32_t)));
+        CK(cudaMemset(d_mx, 0, sizeof(uint32_t)));
+        max_id_kernel<<<1024, 256>>>(g->d_adj, ne, d_mx);
+        CK(cudaGetLastError());
+        uint32_t mx = 0;
+        CK(cudaMemcpy(&mx, d_mx, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+        cudaFree(d_mx);
+        if (mx >= nv) fail(IBFS_E_INVALID, "adjacency id >= nv");
+      }
+      finish_graph(g);
+    } catch (...) {
+      graph_release(g);
+      throw;
+    }
+    *out_graph = g;
+  });
+}
+
+extern "C" int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const uint32_t *u,
+                               const uint32_t *v, int directed, ibfs_graph **out_graph) {
+  return guarded([&] {
+    if (!out_graph) fail(IBFS_E_INVALID, "out_graph is NULL");
+    *out_graph = nullptr;
+    if (nv == 0) fail(IBFS_E_INVALID, "nv must be >= 1");
+    if (n_tuples > 0 && (!u || !v)) fail(IBFS_E_INVALID, "u/v is NULL");
+    if (directed) fail(IBFS_E_UNSUPPORTED, "directed graphs are not implemented in this build");
+    if (n_tuples >= (1ull << 39)) fail(IBFS_E_INVALID, "too many tuples");
+    DeviceScope ds(device);
+    const uint64_t ne = 2 * n_tuples;
+    ibfs_graph *g = new ibfs_graph();
+    std::vector<void *> tmp;
+    auto dalloc = [&](size_t bytes) {
+      void *p = nullptr;
+      CK(cudaMalloc(&p, std::max<size_t>(bytes, 256)));
+      tmp.push_back(p);
+      return p;
+    };
+    try {
+      g->device = device;
+      g->nv = nv;
+      g->ne = ne;
+      uint32_t *d_u = (uint32_t *)dalloc(n_tuples * 4), *d_v = (uint32_t *)dalloc(n_tuples * 4);
+      if (n_tuples) {
+        CK(cudaMemcpy(d_u, u, n_tuples * 4, cudaMemcpyDefault));
+        CK(cudaMemcpy(d_v, v, n_tuples * 4, cudaMemcpyDefault));
+      }
+      uint32_t *keys_a = (uint32_t *)dalloc(ne * 4), *keys_b = (uint32_t *)dalloc(ne * 4);
+      uint32_t *vals_a = (uint32_t *)dalloc(ne * 4);
+      unsigned long long *deg = (unsigned long long *)dalloc(((size_t)nv + 1) * 8);
+      uint32_t *bad = (uint32_t *)dalloc(4);
+      CK(cudaMemset(deg, 0, ((size_t)nv + 1) * 8));
+      CK(cudaMemset(bad, 0, 4));
+      if (n_tuples) {
+        explode_kernel<<<4096, 256>>>(d_u, d_v, n_tuples, keys_a, vals_a, deg, nv, bad);
+        CK(cudaGetLastError());
+      }
+      uint32_t hbad = 0;
+      CK(cudaMemcpy(&hbad, bad, 4, cudaMemcpyDeviceToHost));
+      if (hbad) fail(IBFS_E_INVALID, "tuple vertex id >= nv");
+      cudaFree(d_u);
+      cudaFree(d_v);
+      tmp[0] = tmp[1] = nullptr;
+      CK(cudaMalloc(&g->d_off, ((size_t)nv + 1) * sizeof(unsigned long long)));
+      {  // offsets = exclusive scan of degrees (deg[nv] = 0 gives offsets[nv] = ne)
+        size_t tb = 0;
+        CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, g->d_off, (int64_t)nv + 1));
+        void *t = dalloc(tb);
+        CK(cub::DeviceScan::ExclusiveSum(t, tb, deg, g->d_off, (int64_t)nv + 1));
+      }
+      CK(cudaMalloc(&g->d_adj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
+      if (ne) {  // stable radix sort of (src, dst) by src keeps tuple order within rows
+        int bits = 1;
+        while (bits < 32 && (1ull << bits) < nv) ++bits;
+        size_t tb = 0;
+        CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, keys_a, keys_b, vals_a, g->d_adj, (int64_t)ne, 0, bits));
+        void *t = dalloc(tb);
+        CK(cub::DeviceRadixSort::SortPairs(t, tb, keys_a, keys_b, vals_a, g->d_adj, (int64_t)ne, 0, bits));
+      }
+      CK(cudaDeviceSynchronize());
+      g->h_off.resize((size_t)nv + 1);
+      CK(cudaMemcpy(g->h_off.data(), g->d_off, ((size_t)nv + 1) * 8, cudaMemcpyDeviceToHost));
+      for (void *p : tmp) cudaFree(p);
+      tmp.clear();
+      finish_graph(g);
+    } catch (...) {
+      for (void *p : tmp) cudaFree(p);
+      graph_release(g);
+      throw;
+    }
+    *out_graph = g;
+  });
+}
+
+extern "C" int ibfs_graph_info(const ibfs_graph *g, uint32_t *nv, uint64_t *ne, uint32_t *max_degree,
+                               int *device) {
+  return guarded([&] {
+    if (!g) fail(IBFS_E_INVALID, "graph is NULL");
+    if (nv) *nv = g->nv;
+    if (ne) *ne = g->ne;
+    if (max_degree) *max_degree = g->max_deg;
+    if (device) *device = g->device;
+  });
+}
+
+extern "C" int ibfs_graph_export_csr(const ibfs_graph *g, uint64_t *offsets, uint32_t *adj) {
+  return guarded([&] {
+    if (!g || !offsets || (g->ne && !adj)) fail(IBFS_E_INVALID, "NULL argument");
+    DeviceScope ds(g->device);
+    CK(cudaMemcpy(offsets, g->d_off, ((size_t)g->nv + 1) * 8, cudaMemcpyDeviceToHost));
+    if (g->ne) CK(cudaMemcpy(adj, g->d_adj, g->ne * 4, cudaMemcpyDeviceToHost));
+  });
+}
+
+extern "C" void ibfs_free(ibfs_graph *g) { graph_release(g); }
+
+extern "C" int ibfs_set_allocator(void *(*alloc)(size_t, int, void *), void (*release)(void *, int, void *),
+                                  void *ctx) {
+  return guarded([&] {
+    if ((alloc == nullptr) != (release == nullptr)) fail(IBFS_E_INVALID, "alloc and release must both be set or both NULL");
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    g_alloc.alloc = alloc;
+    g_alloc.release = release;
+    g_alloc.ctx = ctx;
+  });
+}
+
+// ----------------------------------------------------------------------- planning ----
+namespace {
+// hub[r] per DESIGN.md reading #16: the neighbour w of sources[r] with deg(w) > q (any
+// degree if `uniform`) maximising (deg(w), -w); 0xffffffff if none.  One warp per source.
+__global__ void hub_kernel(const unsigned long long *off, const uint32_t *adj, const uint32_t *deg,
+                           const uint32_t *src, uint32_t n, uint32_t q, int uniform, uint32_t *hub,
+                           uint32_t *sdeg) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t warps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < n; r += warps) {
+    const uint32_t s = src[r];
+    const unsigned long long e0 = off[s], e1 = off[s + 1];
+    unsigned long long best = 0;
+    bool have = false;
+    for (unsigned long long e = e0 + lane; e < e1; e += 32) {
+      const uint32_t w = adj[e];
+      const uint32_t dw = deg[w];
+      if (uniform || dw > q) {
+        const unsigned long long key = ((unsigned long long)dw << 32) | (0xffffffffu - w);
+        if (!have || key > best) { best = key; have = true; }
+      }
+    }
+    // warp max over (have, best)
+    unsigned long long k = have ? best + 1 : 0;  // +1 keeps "none" = 0 distinct
+    for (int o = 16; o > 0; o >>= 1) {
+      unsigned long long y = __shfl_xor_sync(FULL, k, o);
+      k = y > k ? y : k;
+    }
+    if (lane == 0) {
+      hub[r] = k ? (0xffffffffu - (uint32_t)((k - 1) & 0xffffffffull)) : 0xffffffffu;
+      sdeg[r] = deg[s];
+    }
+  }
+}
+}  // namespace
+
+extern "C" void ibfs_plan_params_default(ibfs_plan_params *p) {
+  if (!p) return;
+  std::memset(p, 0, sizeof(*p));
+  p->mode = 0;
+  p->q = 128;
+  p->n_p = 4;
+  p->p[0] = 4; p->p[1] = 16; p->p[2] = 64; p->p[3] = 128;
+  p->hops = 1;
+  p->seed = 3;
+}
+
+extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
+                                uint32_t group_bits, const ibfs_plan_params *params, uint32_t *out_perm,
+                                uint32_t *out_n_groups) {
+  return guarded([&] {
+    if (!g) fail(IBFS_E_INVALID, "graph is NULL");
+    if (group_bits != 32 && group_bits != 64 && group_bits != 128) fail(IBFS_E_INVALID, "group_bits must be 32, 64 or 128");
+    if (n > 0 && (!sources || !out_perm)) fail(IBFS_E_INVALID, "sources/out_perm is NULL");
+    ibfs_plan_params pp;
+    if (params) pp = *params; else ibfs_plan_params_default(&pp);
+    if (pp.mode > 2) fail(IBFS_E_INVALID, "plan mode must be 0, 1 or 2");
+    if (pp.mode == 0 && (pp.n_p < 1 || pp.n_p > 8)) fail(IBFS_E_INVALID, "n_p must be 1..8");
+    if (pp.mode == 0 && pp.hops != 1) fail(IBFS_E_UNSUPPORTED, "only hops = 1 is implemented");
+    if (out_n_groups) *out_n_groups = (n + group_bits - 1) / group_bits;
+    if (n == 0) return;
+    std::vector<uint32_t> hsrc(n);
+    DeviceScope ds(g->device);
+    CK(cudaMemcpy(hsrc.data(), sources, (size_t)n * 4, cudaMemcpyDefault));
+    for (uint32_t r = 0; r < n; ++r)
+      if (hsrc[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
+    std::vector<uint32_t> hub(n, 0xffffffffu), sdeg(n, 0);
+    if (pp.mode == 0) {
+      uint32_t *d_src = nullptr, *d_hub = nullptr, *d_sdeg = nullptr;
+      CK(cudaMalloc(&d_src, (size_t)n * 4));
+      CK(cudaMalloc(&d_hub, (size_t)n * 4));
+      CK(cudaMalloc(&d_sdeg, (size_t)n * 4));
+      CK(cudaMemcpy(d_src, hsrc.data(), (size_t)n * 4, cudaMemcpyHostToDevice));
+      const int uniform = g->max_deg <= pp.q ? 1 : 0;
+      uint32_t blocks = std::min<uint32_t>((n + 7) / 8, 65535u);
+      hub_kernel<<<blocks, 256>>>(g->d_off, g->d_adj, g->d_deg, d_src, n, pp.q, uniform, d_hub, d_sdeg);
+      cudaError_t e = cudaGetLastError();
+      if (e == cudaSuccess) e = cudaMemcpy(hub.data(), d_hub, (size_t)n * 4, cudaMemcpyDeviceToHost);
+      if (e == cudaSuccess) e = cudaMemcpy(sdeg.data(), d_sdeg, (size_t)n * 4, cudaMemcpyDeviceToHost);
+      cudaFree(d_src);
+      cudaFree(d_hub);
+      cudaFree(d_sdeg);
+      CK(e);
+    }
+    auto deg_of = [&](uint32_t x) -> uint64_t { return g->h_off[x + 1] - g->h_off[x]; };
+    ibfs::plan::make_plan(pp, group_bits, n, hub, sdeg, deg_of, out_perm);
+  });
+}
+
+// ---------------------------------------------------------------------- traversal ----
+extern "C" void ibfs_run_opts_default(ibfs_run_opts *o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof(*o));
+  o->direction = IBFS_DIR_AUTO;
+  o->bu_from = 2;
+  o->alpha = 4.0f;
+  o->beta = 24.0f;
+}
+
+namespace {
+
+constexpr int LEVELS_PER_CHECK = 2;
+
+struct EventTimer {
+  std::vector<cudaEvent_t> ev;
+  size_t used = 0;
+  ~EventTimer() {
+    for (auto e : ev) cudaEventDestroy(e);
+  }
+  cudaEvent_t next() {
+    if (used == ev.size()) {
+      cudaEvent_t e;
+      CK(cudaEventCreate(&e));
+      ev.push_back(e);
+    }
+    return ev[used++];
+  }
+};
+
+template <typename T>
+void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t *out_depths,
+               const ibfs_run_opts &o, ibfs_stats *stats) {
+  constexpr int W = WordBits<T>::value;
+  constexpr size_t B = sizeof(T);
+  cudaStream_t stream = (cudaStream_t)o.cuda_stream;
+  const uint32_t nv = g->nv;
+  const uint32_t n_groups = (n + W - 1) / W;
+  const bool out_dev = is_device_ptr(out_depths);
+  const bool out_host = out_depths && !out_dev;
+
+  // groups per launch batch
+  uint32_t G = o.groups_in_flight;
+  if (G == 0) {
+    uint64_t want = (4ull << 20) / std::max<uint32_t>(nv, 1) + 1;
+    G = (uint32_t)std::min<uint64_t>(want, MAX_G);
+  }
+  G = std::max<uint32_t>(1, std::min<uint32_t>({G, (uint32_t)MAX_G, n_groups}));
+  const size_t gstride = ((size_t)nv + 15) & ~(size_t)15;
+  const size_t rows_bytes_per_group = (size_t)W * nv;
+  size_t free_b = 0, total_b = 0;
+  CK(cudaMemGetInfo(&free_b, &total_b));
+  auto need = [&](uint32_t gg) {
+    return gg * (3 * gstride * B + (out_dev ? 0 : rows_bytes_per_group)) + (size_t)n * 24;
+  };
+  while (G > 1 && need(G) > free_b / 10 * 8) G = (G + 1) / 2;
+
+  Scratch sc(g->device, stream);
+  uint32_t *d_src = sc.get<uint32_t>(n);
+  CK(cudaMemcpyAsync(d_src, sources, (size_t)n * 4, cudaMemcpyDefault, stream));
+  T *visited = sc.get<T>(G * gstride);
+  T *buf0 = sc.get<T>(G * gstride);
+  T *buf1 = sc.get<T>(G * gstride);
+  GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
+  LevelStat *lstat = sc.get<LevelStat>((size_t)G * MAXL);
+  uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
+  uint32_t *flags = sc.get<uint32_t>(2);  // batch_done, range_err
+  unsigned long long *d_m = sc.get<unsigned long long>((size_t)G * W);
+  unsigned long long *d_dig = sc.get<unsigned long long>((size_t)G * W);
+  int8_t *staging = out_dev ? nullptr : sc.get<int8_t>((size_t)G * rows_bytes_per_group);
+  CK(cudaMemsetAsync(flags, 0, 8, stream));
+
+  HostPinned pin(4096);
+  volatile uint32_t *h_done = (volatile uint32_t *)pin.p;  // [0..255] done slots, [256] range
+  std::vector<LevelStat> h_lstat((size_t)G * MAXL);
+  std::vector<unsigned long long> h_m((size_t)G * W), h_dig((size_t)G * W);
+
+  BatchArgs<T> a{};
+  a.off = g->d_off;
+  a.adj = g->d_adj;
+  a.deg = g->d_deg;
+  a.nv = nv;
+  a.gstride = gstride;
+  a.visited = visited;
+  a.buf0 = buf0;
+  a.buf1 = buf1;
+  a.ctrl = ctrl;
+  a.lstat = lstat;
+  a.work_ctr = work_ctr;
+  a.batch_done = flags;
+  a.range_err = flags + 1;
+  a.n_total = n;
+  a.chunks = g->d_chunks;
+  a.n_chunks = g->n_chunks;
+  a.tile_begin = g->d_tiles;
+  a.n_tiles = g->n_tiles;
+  a.pol.mode = o.direction;
+  a.pol.bu_from = o.bu_from;
+  a.pol.alpha = o.alpha;
+  a.pol.beta = o.beta;
+  a.pol.nv_active = g->nv_active;
+  a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
+  for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
+  uint32_t first_dir = 0;
+  if (o.direction == IBFS_DIR_BU_FROM) first_dir = o.bu_from <= 1 ? 1 : 0;
+  if (o.direction == IBFS_DIR_SCHEDULE && a.pol.sched_len > 0) first_dir = a.pol.sched[0];
+
+  const int expand_grid = g->num_sms * g->expand_blocks_per_sm;
+  EventTimer timer;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, kexp, kcom, kinit;
+  std::vector<cudaEvent_t> chk(256);
+  for (auto &e : chk) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  struct EvGuard {
+    std::vector<cudaEvent_t> &v;
+    ~EvGuard() {
+      for (auto e : v) cudaEventDestroy(e);
+    }
+  } evg{chk};
+
+  ibfs_stats st{};
+  uint64_t launches = 0;
+  bool range_error = false;
+  std::vector<ibfs_level_stats> per_level(MAXL);
+
+  for (uint32_t gb0 = 0; gb0 < n_groups; gb0 += G) {
+    const uint32_t Gb = std::min(G, n_groups - gb0);
+    a.G = (int)Gb;
+    a.group0 = gb0;
+    a.src = d_src + (size_t)gb0 * W;
+    a.out = out_dev ? out_depths + (size_t)gb0 * rows_bytes_per_group : staging;
+    const uint32_t rows_in_batch = std::min<uint32_t>(Gb * W, n - gb0 * W);
+    CK(cudaMemsetAsync(flags, 0, 4, stream));
+    cudaEvent_t w0 = timer.next(), w1 = timer.next();
+    CK(cudaEventRecord(w0, stream));
+    {
+      cudaEvent_t i0 = nullptr, i1 = nullptr;
+      if (o.timing) { i0 = timer.next(); i1 = timer.next(); CK(cudaEventRecord(i0, stream)); }
+      uint32_t bx = (uint32_t)std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, std::max<uint32_t>(1, 2048 / Gb));
+      init_state_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a);
+      init_sources_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
+      CK(cudaGetLastError());
+      launches += 2;
+      st.init_launches += 2;
+      st.init_bytes += (uint64_t)Gb * (3 * nv * B) + (uint64_t)rows_in_batch * nv;
+      if (o.timing) { CK(cudaEventRecord(i1, stream)); kinit.push_back({i0, i1}); }
+    }
+    const uint32_t commit_bx = (uint32_t)std::max<uint64_t>(
+        1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, (uint64_t)g->num_sms * 8 / Gb));
+    int level = 1;
+    int chunk = 0;
+    int last_level_launched = 0;
+    while (level <= MAXL - 1) {
+      const int lend = std::min(level + LEVELS_PER_CHECK, MAXL);
+      for (int l = level; l < lend; ++l) {
+        cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
+        if (o.timing) { e0 = timer.next(); e1 = timer.next(); e2 = timer.next(); CK(cudaEventRecord(e0, stream)); }
+        expand_kernel<T><<<expand_grid, BLOCK, 0, stream>>>(a, l);
+        if (o.timing) CK(cudaEventRecord(e1, stream));
+        commit_kernel<T><<<dim3(commit_bx, Gb), BLOCK, 0, stream>>>(a, l);
+        if (o.timing) { CK(cudaEventRecord(e2, stream)); kexp.push_back({e0, e1}); kcom.push_back({e1, e2}); }
+        launches += 2;
+        st.expand_launches++;
+        st.commit_launches++;
+      }
+      CK(cudaGetLastError());
+      last_level_launched = lend - 1;
+      if (chunk >= 256) fail(IBFS_E_CUDA, "level loop overflow");
+      CK(cudaMemcpyAsync((void *)(h_done + chunk), flags, 4, cudaMemcpyDeviceToHost, stream));
+      CK(cudaEventRecord(chk[chunk], stream));
+      ++chunk;
+      level = lend;
+      if (chunk >= 2) {
+        CK(cudaEventSynchronize(chk[chunk - 2]));
+        if (h_done[chunk - 2] >= Gb) break;
+      }
+    }
+    (void)last_level_launched;
+    CK(cudaEventRecord(w1, stream));
+    win.push_back({w0, w1});
+    // range check (a level-128 discovery means a depth > 127)
+    CK(cudaMemcpyAsync((void *)(h_done + 256), flags + 1, 4, cudaMemcpyDeviceToHost, stream));
+    // finalize: m_s and digests (outside the traversal window)
+    CK(cudaMemsetAsync(d_m, 0, (size_t)G * W * 8, stream));
+    {
+      uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, 2048 / Gb));
+      msum_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a, d_m);
+    }
+    if (stats && stats->per_source_digest) {
+      CK(cudaMemsetAsync(d_dig, 0, (size_t)G * W * 8, stream));
+      uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, 64));
+      digest_kernel<T><<<dim3(bx, Gb * W), BLOCK, 0, stream>>>(a, d_dig);
+    }
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(h_lstat.data(), lstat, (size_t)Gb * MAXL * sizeof(LevelStat), cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(h_m.data(), d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
+    if (stats && stats->per_source_digest)
+      CK(cudaMemcpyAsync(h_dig.data(), d_dig, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
+    if (out_host) {
+      cudaEvent_t c0 = timer.next(), c1 = timer.next();
+      CK(cudaEventRecord(c0, stream));
+      CK(cudaMemcpyAsync(out_depths + (size_t)gb0 * rows_bytes_per_group, staging,
+                         (size_t)rows_in_batch * nv, cudaMemcpyDeviceToHost, stream));
+      CK(cudaEventRecord(c1, stream));
+      CK(cudaStreamSynchronize(stream));
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, c0, c1));
+      st.copyout_ms += ms;
+    }
+    CK(cudaStreamSynchronize(stream));
+    if (h_done[256]) range_error = true;
+    // accumulate per-source outputs and statistics
+    for (uint32_t r = 0; r < rows_in_batch; ++r) {
+      st.edges_traversed += h_m[r];
+      if (stats && stats->per_source_m) stats->per_source_m[(size_t)gb0 * W + r] = h_m[r];
+      if (stats && stats->per_source_digest) stats->per_source_digest[(size_t)gb0 * W + r] = h_dig[r];
+    }
+    for (uint32_t gi = 0; gi < Gb; ++gi) {
+      for (int l = 1; l < MAXL; ++l) {
+        const LevelStat &L = h_lstat[(size_t)gi * MAXL + l];
+        if (L.dir == 0) continue;
+        ibfs_level_stats &P = per_level[l - 1];
+        const bool td = L.dir == 1;
+        st.max_levels = std::max<uint32_t>(st.max_levels, (uint32_t)l);
+        if (td) { P.td_groups++; P.jfq_td += L.jfq; P.fq_td += L.fq; st.levels_td++; st.sd_fq_td += L.fq; st.sd_jfq_td += L.jfq; }
+        else { P.bu_groups++; P.jfq_bu += L.jfq; P.fq_bu += L.fq; st.levels_bu++; st.sd_fq_bu += L.fq; st.sd_jfq_bu += L.jfq; }
+        P.inspected += L.insp;
+        P.new_pairs += L.newp;
+        st.edges_inspected += L.insp;
+        // DESIGN.md §5 byte model
+        uint64_t eb = (uint64_t)nv * B + 4 * L.jfq + 8 * L.proc + (4 + B) * L.insp + B * L.writes;
+        uint64_t cb = (uint64_t)nv * (3 * B + 4) + B * L.nf + L.newp;
+        st.expand_bytes += eb;
+        st.commit_bytes += cb;
+      }
+    }
+  }
+  if (range_error) fail(IBFS_E_RANGE, "a depth exceeds 127 (int8 output)");
+  // times
+  for (auto &p : win) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.traverse_ms += ms; }
+  for (auto &p : kexp) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.expand_ms += ms; }
+  for (auto &p : kcom) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.commit_ms += ms; }
+  for (auto &p : kinit) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.init_ms += ms; }
+  st.n_groups = n_groups;
+  st.n_launches = launches;
+  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes;
+  if (stats) {
+    st.per_source_m = stats->per_source_m;
+    st.per_source_digest = stats->per_source_digest;
+    st.level_cap = stats->level_cap;
+    st.per_level = stats->per_level;
+    if (st.per_level)
+      for (uint32_t i = 0; i < st.level_cap; ++i) st.per_level[i] = i < (uint32_t)MAXL ? per_level[i] : ibfs_level_stats{};
+    *stats = st;
+  }
+}
+
+}  // namespace
+
+extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_t n, uint32_t group_bits,
+                           int8_t *out_depths, const ibfs_run_opts *opts, ibfs_stats *stats) {
+  return guarded([&] {
+    if (!g) fail(IBFS_E_INVALID, "graph is NULL");
+    if (group_bits != 32 && group_bits != 64 && group_bits != 128) fail(IBFS_E_INVALID, "group_bits must be 32, 64 or 128");
+    if (n > 0 && !sources) fail(IBFS_E_INVALID, "sources is NULL");
+    ibfs_run_opts o;
+    if (opts) o = *opts; else ibfs_run_opts_default(&o);
+    if (o.direction > 3) fail(IBFS_E_INVALID, "bad direction mode");
+    if (o.direction == IBFS_DIR_SCHEDULE && o.schedule_len > 0 && !o.schedule) fail(IBFS_E_INVALID, "schedule is NULL");
+    if (!(o.alpha > 0) || !(o.beta > 0)) fail(IBFS_E_INVALID, "alpha and beta must be > 0");
+    if (stats) {
+      if (stats->per_source_m) std::memset(stats->per_source_m, 0, (size_t)n * 8);
+      if (stats->per_source_digest) std::memset(stats->per_source_digest, 0, (size_t)n * 8);
+    }
+    if (n == 0) {
+      if (stats) {
+        ibfs_stats z{};
+        z.per_source_m = stats->per_source_m;
+        z.per_source_digest = stats->per_source_digest;
+        z.level_cap = stats->level_cap;
+        z.per_level = stats->per_level;
+        if (z.per_level) std::memset(z.per_level, 0, sizeof(ibfs_level_stats) * z.level_cap);
+        *stats = z;
+      }
+      return;
+    }
+    DeviceScope ds(g->device);
+    // sources: validate on the host
+    std::vector<uint32_t> hs(n);
+    CK(cudaMemcpy(hs.data(), sources, (size_t)n * 4, cudaMemcpyDefault));
+    for (uint32_t r = 0; r < n; ++r)
+      if (hs[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
+    if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), n, out_depths, o, stats);
+    else if (group_bits == 64) run_typed<unsigned long long>(g, hs.data(), n, out_depths, o, stats);
+    else run_typed<u128>(g, hs.data(), n, out_depths, o, stats);
+  });
+}
+
+extern "C" int ibfs_run(const ibfs_graph *g, const uint32_t *sources, uint32_t n, uint32_t group_bits,
+                        int8_t *out_depths) {
+  return ibfs_run_ex(g, sources, n, group_bits, out_depths, nullptr, nullptr);
+}

@@ -7,7 +7,8 @@
  * Recipe (SURVEY.md §8(d) "Generator spec"):
  *   - tuple e in [0, M), M = ef * 2^scale; for each bit b in [0, scale) one 64-bit
  *     counter-based draw h = mix64(mix64(seed + GOLDEN) ^ ((e << 6) | b)) gives two
- *     32-bit uniforms r1 = hi32(h) / 2^32, r2 = lo32(h) / 2^32;
+ *     32-bit uniforms r1 = hi32(h) / 2^32, r2 = lo32(h) / 2^32 (compared exactly as
+ *     integers against floor(p * 2^32));
  *     ii = r1 > A+B, jj = r2 > (ii ? C/(C+D) : A/(A+B)); u |= ii << b, v |= jj << b.
  *     The quadrant probabilities are then A, B, C, D (PAPER.md P:L975 gives
  *     (A,B,C) = (0.57,0.19,0.19) for the Graph500 "KG" graphs and (0.45,0.15,0.15)
@@ -44,22 +45,20 @@ typedef struct {
   uint64_t e0, e1;
   int scale;
   uint64_t key;
-  double ab, c_cd, a_ab;
+  uint64_t t_ab, t_c_cd, t_a_ab; /* floor(p * 2^32): r > p  <=>  (r * 2^32) > floor(p * 2^32) */
   uint32_t *u, *v;
   const uint32_t *perm;
 } rmat_job;
 
 static void *rmat_worker(void *arg) {
   rmat_job *j = (rmat_job *)arg;
-  const double inv32 = 1.0 / 4294967296.0;
   for (uint64_t e = j->e0; e < j->e1; ++e) {
     uint32_t u = 0, v = 0;
     for (int b = 0; b < j->scale; ++b) {
       uint64_t h = mix64(j->key ^ ((e << 6) | (uint64_t)b));
-      double r1 = (double)(uint32_t)(h >> 32) * inv32;
-      double r2 = (double)(uint32_t)(h & 0xffffffffULL) * inv32;
-      uint32_t ii = r1 > j->ab;
-      uint32_t jj = r2 > (ii ? j->c_cd : j->a_ab);
+      uint64_t r1 = h >> 32, r2 = h & 0xffffffffULL;
+      uint32_t ii = r1 > j->t_ab;
+      uint32_t jj = r2 > (ii ? j->t_c_cd : j->t_a_ab);
       u |= ii << b;
       v |= jj << b;
     }
@@ -68,6 +67,14 @@ static void *rmat_worker(void *arg) {
     j->v[e] = v;
   }
   return NULL;
+}
+
+/* floor(p * 2^32) as an integer threshold (exact: for integer r, r > x <=> r > floor(x)). */
+static uint64_t thresh(double p) {
+  double x = p * 4294967296.0;
+  if (x >= 4294967296.0) return 4294967296ULL;
+  if (x <= 0) return 0;
+  return (uint64_t)x;
 }
 
 /* Fisher-Yates permutation of [0, n): out[i] = pi(i). */
@@ -105,9 +112,9 @@ int ibfs_gen_rmat(int scale, uint32_t edgefactor, double A, double B, double C,
     jobs[t].e1 = m * (uint64_t)(t + 1) / (uint64_t)threads;
     jobs[t].scale = scale;
     jobs[t].key = key;
-    jobs[t].ab = A + B;
-    jobs[t].c_cd = C / (C + D);
-    jobs[t].a_ab = A / (A + B);
+    jobs[t].t_ab = thresh(A + B);
+    jobs[t].t_c_cd = thresh(C / (C + D));
+    jobs[t].t_a_ab = thresh(A / (A + B));
     jobs[t].u = u;
     jobs[t].v = v;
     jobs[t].perm = perm;

@@ -169,7 +169,7 @@ typedef struct {
   uint64_t sd_fq_td, sd_jfq_td, sd_fq_bu, sd_jfq_bu;  /* Eq. 1 numerators/denominators */
   uint32_t n_groups, max_levels;
   uint32_t levels_td, levels_bu;  /* group-levels run in each direction */
-  uint64_t n_launches;            /* kernels launched inside traverse_ms */
+  uint64_t n_launches;            /* kernels this call launched (traversal + finalize) */
   /* per-kernel device time and algorithmic bytes (bytes always; ms only if opts.timing) */
   double expand_ms, commit_ms, init_ms;
   uint64_t expand_launches, commit_launches, init_launches;

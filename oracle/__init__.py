@@ -48,7 +48,7 @@ def _load():
         lib = ctypes.CDLL(_SO)
         P = ctypes.c_void_p
         lib.oracle_graph_new.restype = P
-        lib.oracle_graph_new.argtypes = [ctypes.c_uint64, ctypes.c_uint64, P, P, ctypes.c_int]
+        lib.oracle_graph_new.argtypes = [ctypes.c_uint64, ctypes.c_uint64, P, P, ctypes.c_int, ctypes.c_int]
         lib.oracle_graph_free.restype = None
         lib.oracle_graph_free.argtypes = [P]
         lib.oracle_graph_nv.restype = ctypes.c_uint64
@@ -76,14 +76,16 @@ class OracleResult:
 class OracleGraph:
     """Adjacency lists built from the raw tuples (never from the GPU path's CSR)."""
 
-    def __init__(self, nv: int, u: np.ndarray, v: np.ndarray, directed: bool = False):
+    def __init__(self, nv: int, u: np.ndarray, v: np.ndarray, directed: bool = False,
+                 threads: int | None = None):
         lib = _load()
         self._u = np.ascontiguousarray(u, dtype=np.uint32)
         self._v = np.ascontiguousarray(v, dtype=np.uint32)
         self.nv = int(nv)
         self.directed = bool(directed)
         self._h = lib.oracle_graph_new(self.nv, int(self._u.shape[0]), self._u.ctypes.data,
-                                       self._v.ctypes.data, 1 if directed else 0)
+                                       self._v.ctypes.data, 1 if directed else 0,
+                                       int(threads or os.cpu_count() or 1))
         if not self._h:
             raise ValueError("oracle_graph_new failed (bad vertex id or out of memory)")
         del self._u, self._v

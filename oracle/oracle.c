@@ -50,29 +50,70 @@ void oracle_graph_free(oracle_graph *g) {
   free(g);
 }
 
-/* Build adjacency lists from the raw tuples, keeping tuple order within each list. */
+/* Build adjacency lists from the raw tuples, keeping tuple order within each list.
+ * Thread t owns the vertex range [lo_t, hi_t) and scans every tuple twice (count, then
+ * fill), appending only to its own lists -- the same sequential append order as a
+ * single pass, just split by owner. */
+typedef struct {
+  uint64_t lo, hi, m;
+  const uint32_t *u, *v;
+  int directed, pass;
+  uint64_t *off;   /* pass 0: counts at off[x + 1]; pass 1: fill cursors */
+  uint32_t *adj;
+} build_job;
+
+static void *build_worker(void *arg) {
+  build_job *j = (build_job *)arg;
+  const uint64_t lo = j->lo, hi = j->hi;
+  for (uint64_t e = 0; e < j->m; ++e) {
+    uint32_t a = j->u[e], b = j->v[e];
+    if (a >= lo && a < hi) {
+      if (j->pass == 0) j->off[a + 1]++;
+      else j->adj[j->off[a]++] = b;
+    }
+    if (!j->directed && b >= lo && b < hi) {
+      if (j->pass == 0) j->off[b + 1]++;
+      else j->adj[j->off[b]++] = a;
+    }
+  }
+  return NULL;
+}
+
 oracle_graph *oracle_graph_new(uint64_t nv, uint64_t m, const uint32_t *u, const uint32_t *v,
-                               int directed) {
+                               int directed, int threads) {
   oracle_graph *g = (oracle_graph *)calloc(1, sizeof(oracle_graph));
   if (!g) return NULL;
   g->nv = nv;
+  for (uint64_t e = 0; e < m; ++e)
+    if (u[e] >= nv || v[e] >= nv) { free(g); return NULL; }
   g->off = (uint64_t *)calloc(nv + 1, sizeof(uint64_t));
   uint64_t entries = directed ? m : 2 * m;
   g->adj = (uint32_t *)malloc((entries ? entries : 1) * sizeof(uint32_t));
-  uint64_t *fill = (uint64_t *)calloc(nv + 1, sizeof(uint64_t));
-  if (!g->off || !g->adj || !fill) { free(fill); oracle_graph_free(g); return NULL; }
-  for (uint64_t e = 0; e < m; ++e) {
-    if (u[e] >= nv || v[e] >= nv) { free(fill); oracle_graph_free(g); return NULL; }
-    g->off[u[e] + 1]++;
-    if (!directed) g->off[v[e] + 1]++;
+  uint64_t *cur = (uint64_t *)malloc((nv + 1) * sizeof(uint64_t));
+  if (!g->off || !g->adj || !cur) { free(cur); oracle_graph_free(g); return NULL; }
+  if (threads < 1) threads = 1;
+  if (threads > 256) threads = 256;
+  if ((uint64_t)threads > nv) threads = (int)nv;
+  pthread_t tid[256];
+  build_job jobs[256];
+  for (int pass = 0; pass < 2; ++pass) {
+    if (pass == 1) {
+      for (uint64_t x = 0; x < nv; ++x) g->off[x + 1] += g->off[x];
+      memcpy(cur, g->off, (nv + 1) * sizeof(uint64_t));
+    }
+    for (int t = 0; t < threads; ++t) {
+      jobs[t].lo = nv * (uint64_t)t / (uint64_t)threads;
+      jobs[t].hi = nv * (uint64_t)(t + 1) / (uint64_t)threads;
+      jobs[t].m = m; jobs[t].u = u; jobs[t].v = v;
+      jobs[t].directed = directed; jobs[t].pass = pass;
+      jobs[t].off = pass == 0 ? g->off : cur;
+      jobs[t].adj = g->adj;
+    }
+    for (int t = 1; t < threads; ++t) pthread_create(&tid[t], NULL, build_worker, &jobs[t]);
+    build_worker(&jobs[0]);
+    for (int t = 1; t < threads; ++t) pthread_join(tid[t], NULL);
   }
-  for (uint64_t x = 0; x < nv; ++x) g->off[x + 1] += g->off[x];
-  for (uint64_t x = 0; x <= nv; ++x) fill[x] = g->off[x];
-  for (uint64_t e = 0; e < m; ++e) {
-    g->adj[fill[u[e]]++] = v[e];
-    if (!directed) g->adj[fill[v[e]]++] = u[e];
-  }
-  free(fill);
+  free(cur);
   return g;
 }
 

@@ -748,11 +748,13 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
     {
       uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, 2048 / Gb));
       msum_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a, d_m);
+      launches++;
     }
     if (stats && stats->per_source_digest) {
       CK(cudaMemsetAsync(d_dig, 0, (size_t)G * W * 8, stream));
       uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, 64));
       digest_kernel<T><<<dim3(bx, Gb * W), BLOCK, 0, stream>>>(a, d_dig);
+      launches++;
     }
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(h_lstat.data(), lstat, (size_t)Gb * MAXL * sizeof(LevelStat), cudaMemcpyDeviceToHost, stream));

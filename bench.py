@@ -232,6 +232,7 @@ def main():
     kern = {
         "expand": (sum(s.expand_bytes for s in sts), sum(s.expand_ms for s in sts), sum(s.expand_launches for s in sts)),
         "commit": (sum(s.commit_bytes for s in sts), sum(s.commit_ms for s in sts), sum(s.commit_launches for s in sts)),
+        "depth": (sum(s.depth_bytes for s in sts), sum(s.depth_ms for s in sts), sum(s.depth_launches for s in sts)),
     }
     dom = max(kern, key=lambda k: kern[k][1])
     b, ms, nl = kern[dom]

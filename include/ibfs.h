@@ -71,6 +71,14 @@ int ibfs_load_csr(int device, uint32_t nv, uint64_t ne, const uint64_t *offsets,
 int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const uint32_t *u,
                     const uint32_t *v, int directed, ibfs_graph **out_graph);
 
+/* Row order of the device adjacency (never changes any result):
+ *   IBFS_ROWS_KEEP      keep the loaded order (tuple order for ibfs_load_edges).
+ *   IBFS_ROWS_HUB_FIRST stable-sort every row by neighbour outdegree, descending, so
+ *                       bottom-up inspection (Alg. 1) meets the vertices most
+ *                       likely visited first and terminates early on hot words. */
+enum { IBFS_ROWS_KEEP = 0, IBFS_ROWS_HUB_FIRST = 1 };
+int ibfs_graph_sort_rows(ibfs_graph *g, int order);
+
 /* Graph facts.  Any output pointer may be NULL. */
 int ibfs_graph_info(const ibfs_graph *g, uint32_t *nv, uint64_t *ne, uint32_t *max_degree,
                     int *device);
@@ -157,6 +165,7 @@ typedef struct {
   uint64_t jfq_bu, fq_bu;         /* same for the BU groups (reading #23) */
   uint64_t inspected;             /* neighbour status words read */
   uint64_t new_pairs;             /* (instance, vertex) pairs discovered (depth == l) */
+  double expand_ms, commit_ms;    /* device time of this level's launches (opts.timing) */
 } ibfs_level_stats;
 
 typedef struct {
@@ -171,9 +180,9 @@ typedef struct {
   uint32_t levels_td, levels_bu;  /* group-levels run in each direction */
   uint64_t n_launches;            /* kernels this call launched (traversal + finalize) */
   /* per-kernel device time and algorithmic bytes (bytes always; ms only if opts.timing) */
-  double expand_ms, commit_ms, init_ms;
-  uint64_t expand_launches, commit_launches, init_launches;
-  uint64_t expand_bytes, commit_bytes, init_bytes;
+  double expand_ms, commit_ms, init_ms, depth_ms;
+  uint64_t expand_launches, commit_launches, init_launches, depth_launches;
+  uint64_t expand_bytes, commit_bytes, init_bytes, depth_bytes;
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */
   uint64_t *per_source_digest;  /* [n] sum over reached v of splitmix64((v<<8)|(d+1)) */

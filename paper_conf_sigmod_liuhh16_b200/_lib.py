@@ -9,7 +9,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-SO = os.path.join(HERE, "libibfs.so")
+SO = os.environ.get("IBFS_LIB") or os.path.join(HERE, "libibfs.so")  # IBFS_LIB: A/B builds
 
 IBFS_OK = 0
 IBFS_E_INVALID = -1
@@ -23,8 +23,9 @@ DIR_AUTO, DIR_TD_ONLY, DIR_BU_FROM, DIR_SCHEDULE = 0, 1, 2, 3
 EXPORTS = [
     "ibfs_version", "ibfs_last_error", "ibfs_load_csr", "ibfs_load_edges", "ibfs_graph_info",
     "ibfs_graph_export_csr", "ibfs_free", "ibfs_plan_params_default", "ibfs_plan_groups",
-    "ibfs_run", "ibfs_run_opts_default", "ibfs_run_ex", "ibfs_set_allocator",
+    "ibfs_run", "ibfs_run_opts_default", "ibfs_run_ex", "ibfs_set_allocator", "ibfs_graph_sort_rows",
 ]
+ROWS_KEEP, ROWS_HUB_FIRST = 0, 1
 
 
 class PlanParams(C.Structure):
@@ -42,7 +43,8 @@ class RunOpts(C.Structure):
 class LevelStats(C.Structure):
     _fields_ = [("td_groups", C.c_uint32), ("bu_groups", C.c_uint32), ("jfq_td", C.c_uint64),
                 ("fq_td", C.c_uint64), ("jfq_bu", C.c_uint64), ("fq_bu", C.c_uint64),
-                ("inspected", C.c_uint64), ("new_pairs", C.c_uint64)]
+                ("inspected", C.c_uint64), ("new_pairs", C.c_uint64),
+                ("expand_ms", C.c_double), ("commit_ms", C.c_double)]
 
 
 class Stats(C.Structure):
@@ -54,9 +56,11 @@ class Stats(C.Structure):
                 ("n_groups", C.c_uint32), ("max_levels", C.c_uint32), ("levels_td", C.c_uint32),
                 ("levels_bu", C.c_uint32), ("n_launches", C.c_uint64),
                 ("expand_ms", C.c_double), ("commit_ms", C.c_double), ("init_ms", C.c_double),
+                ("depth_ms", C.c_double),
                 ("expand_launches", C.c_uint64), ("commit_launches", C.c_uint64),
-                ("init_launches", C.c_uint64),
+                ("init_launches", C.c_uint64), ("depth_launches", C.c_uint64),
                 ("expand_bytes", C.c_uint64), ("commit_bytes", C.c_uint64), ("init_bytes", C.c_uint64),
+                ("depth_bytes", C.c_uint64),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),
                 ("level_cap", C.c_uint32), ("per_level", C.c_void_p)]
 
@@ -89,6 +93,8 @@ def load(path: str | None = None):
     lib.ibfs_graph_info.restype = C.c_int
     lib.ibfs_graph_info.argtypes = [P, C.POINTER(C.c_uint32), C.POINTER(C.c_uint64),
                                     C.POINTER(C.c_uint32), C.POINTER(C.c_int)]
+    lib.ibfs_graph_sort_rows.restype = C.c_int
+    lib.ibfs_graph_sort_rows.argtypes = [P, C.c_int]
     lib.ibfs_graph_export_csr.restype = C.c_int
     lib.ibfs_graph_export_csr.argtypes = [P, P, P]
     lib.ibfs_free.restype = None

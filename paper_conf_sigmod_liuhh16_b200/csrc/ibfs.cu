@@ -13,6 +13,7 @@
 #include <cuda_runtime.h>
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
+#include <cub/device/device_segmented_sort.cuh>
 
 #include <algorithm>
 #include <cmath>
@@ -154,14 +155,6 @@ bool is_device_ptr(const void *p) {
   return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
 }
 
-struct HostPinned {
-  void *p = nullptr;
-  explicit HostPinned(size_t bytes) { CK(cudaMallocHost(&p, bytes)); }
-  ~HostPinned() {
-    if (p) cudaFreeHost(p);
-  }
-};
-
 }  // namespace
 
 // -------------------------------------------------------------------------- graph ----
@@ -176,8 +169,6 @@ struct ibfs_graph {
   uint32_t *d_deg = nullptr;
   HubChunk *d_chunks = nullptr;
   uint32_t n_chunks = 0;
-  uint32_t *d_tiles = nullptr;
-  uint32_t n_tiles = 0;
   std::vector<uint64_t> h_off;  // host copy (tiling, planner)
   int num_sms = 148;
   int expand_blocks_per_sm = 1;
@@ -193,7 +184,6 @@ void graph_release(ibfs_graph *g) {
   cudaFree(g->d_adj);
   cudaFree(g->d_deg);
   cudaFree(g->d_chunks);
-  cudaFree(g->d_tiles);
   if (prev >= 0) cudaSetDevice(prev);
   cudaGetLastError();
   delete g;
@@ -227,48 +217,31 @@ __global__ void max_id_kernel(const uint32_t *adj, unsigned long long ne, uint32
   if ((threadIdx.x & 31) == 0) atomicMax(mx, m);
 }
 
-// Static work decomposition: hub chunks for deg > HUB_T, and tiles of
-// consecutive vertices holding <= V_TILE vertices and <= E_TILE non-hub edges.
+// Static hub decomposition: the rows of vertices with degree > HUB_T are
+// cut into chunks of CHUNK edges, each a work item a whole CTA sweeps.
 void build_decomposition(ibfs_graph *g) {
   std::vector<HubChunk> chunks;
-  std::vector<uint32_t> tiles;
-  tiles.push_back(0);
-  uint64_t cur_e = 0;
-  uint32_t cur_n = 0;
   for (uint32_t v = 0; v < g->nv; ++v) {
-    uint64_t d = g->h_off[v + 1] - g->h_off[v];
-    uint64_t dn = d > (uint64_t)HUB_T ? 0 : d;
-    if (d > (uint64_t)HUB_T) {
-      uint32_t first = 1;
-      for (uint64_t e = g->h_off[v]; e < g->h_off[v + 1]; e += CHUNK) {
-        HubChunk c;
-        c.e0 = e;
-        c.e1 = std::min<uint64_t>(e + CHUNK, g->h_off[v + 1]);
-        c.v = v;
-        c.first = first;
-        first = 0;
-        chunks.push_back(c);
-      }
+    const uint64_t d = g->h_off[v + 1] - g->h_off[v];
+    if (d <= (uint64_t)HUB_T) continue;
+    uint32_t first = 1;
+    for (uint64_t e = g->h_off[v]; e < g->h_off[v + 1]; e += CHUNK) {
+      HubChunk c;
+      c.e0 = e;
+      c.e1 = std::min<uint64_t>(e + CHUNK, g->h_off[v + 1]);
+      c.v = v;
+      c.first = first;
+      first = 0;
+      chunks.push_back(c);
     }
-    if (cur_n > 0 && (cur_n == (uint32_t)V_TILE || cur_e + dn > (uint64_t)E_TILE)) {
-      tiles.push_back(v);
-      cur_n = 0;
-      cur_e = 0;
-    }
-    cur_n++;
-    cur_e += dn;
   }
-  tiles.push_back(g->nv);
-  g->n_tiles = (uint32_t)(tiles.size() - 1);
   g->n_chunks = (uint32_t)chunks.size();
-  CK(cudaMalloc(&g->d_tiles, tiles.size() * sizeof(uint32_t)));
-  CK(cudaMemcpy(g->d_tiles, tiles.data(), tiles.size() * sizeof(uint32_t), cudaMemcpyHostToDevice));
   CK(cudaMalloc(&g->d_chunks, std::max<size_t>(chunks.size(), 1) * sizeof(HubChunk)));
   if (!chunks.empty())
     CK(cudaMemcpy(g->d_chunks, chunks.data(), chunks.size() * sizeof(HubChunk), cudaMemcpyHostToDevice));
 }
 
-// Degrees, max degree, tiles; offsets must be in g->d_off and g->h_off.
+// Degrees, max degree, hub chunks; offsets must be in g->d_off and g->h_off.
 void finish_graph(ibfs_graph *g) {
   CK(cudaMalloc(&g->d_deg, std::max<size_t>(g->nv, 1) * sizeof(uint32_t)));
   unsigned long long *d_stats = nullptr;
@@ -287,8 +260,14 @@ void finish_graph(ibfs_graph *g) {
   build_decomposition(g);
   int dev = g->device;
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev));
+  CK(cudaFuncSetAttribute(expand_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)sizeof(TileQueue<uint32_t>)));
+  CK(cudaFuncSetAttribute(expand_kernel<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)sizeof(TileQueue<unsigned long long>)));
+  CK(cudaFuncSetAttribute(expand_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)sizeof(TileQueue<u128>)));
   int occ = 1;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, expand_kernel<u128>, BLOCK, 0));
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, expand_kernel<u128>, BLOCK, sizeof(TileQueue<u128>)));
   g->expand_blocks_per_sm = std::max(1, occ);
   set_pool_threshold(dev);
 }
@@ -440,6 +419,84 @@ extern "C" int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const
   });
 }
 
+namespace {
+// key = ~deg(w): ascending key order = neighbour degree descending
+__global__ void hubkey_kernel(const uint32_t *adj, const uint32_t *deg, unsigned long long n, uint32_t *keys) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    keys[i] = ~deg[adj[i]];
+}
+__global__ void rel_offsets_kernel(const unsigned long long *off, uint32_t r0, uint32_t nr, int *rel) {
+  const unsigned long long base = off[r0];
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i <= nr; i += gridDim.x * blockDim.x)
+    rel[i] = (int)(off[r0 + i] - base);
+}
+}  // namespace
+
+extern "C" int ibfs_graph_sort_rows(ibfs_graph *g, int order) {
+  return guarded([&] {
+    if (!g) fail(IBFS_E_INVALID, "graph is NULL");
+    if (order != IBFS_ROWS_KEEP && order != IBFS_ROWS_HUB_FIRST) fail(IBFS_E_INVALID, "bad row order");
+    if (order == IBFS_ROWS_KEEP || g->ne == 0) return;
+    DeviceScope ds(g->device);
+    // rows in batches of <= 2^30 entries (CUB segmented sort takes int sizes)
+    const unsigned long long cap = 1ull << 30;
+    unsigned long long maxb = 0;
+    std::vector<std::pair<uint32_t, uint32_t>> batches;
+    uint32_t r0 = 0;
+    while (r0 < g->nv) {
+      uint32_t r1 = r0;
+      while (r1 < g->nv && g->h_off[r1 + 1] - g->h_off[r0] <= cap) ++r1;
+      if (r1 == r0) ++r1;  // a single row longer than cap (degree > 2^30): not expected
+      batches.push_back({r0, r1});
+      maxb = std::max<unsigned long long>(maxb, g->h_off[r1] - g->h_off[r0]);
+      r0 = r1;
+    }
+    if (maxb > 0x7fffffffull) fail(IBFS_E_UNSUPPORTED, "row longer than 2^31 entries");
+    std::vector<void *> tmp;
+    auto dalloc = [&](size_t bytes) {
+      void *p = nullptr;
+      CK(cudaMalloc(&p, std::max<size_t>(bytes, 256)));
+      tmp.push_back(p);
+      return p;
+    };
+    try {
+      uint32_t *kin = (uint32_t *)dalloc(maxb * 4), *kout = (uint32_t *)dalloc(maxb * 4);
+      uint32_t *vout = (uint32_t *)dalloc(maxb * 4);
+      size_t max_rows = 0;
+      for (auto &b : batches) max_rows = std::max<size_t>(max_rows, b.second - b.first);
+      int *rel = (int *)dalloc((max_rows + 1) * 4);
+      size_t tb_max = 0;
+      for (auto &b : batches) {
+        size_t tb = 0;
+        const int nitems = (int)(g->h_off[b.second] - g->h_off[b.first]);
+        const int nseg = (int)(b.second - b.first);
+        CK(cub::DeviceSegmentedSort::StableSortPairs(nullptr, tb, kin, kout, vout, vout, nitems, nseg, rel, rel + 1));
+        tb_max = std::max(tb_max, tb);
+      }
+      void *temp = dalloc(tb_max);
+      for (auto &b : batches) {
+        const unsigned long long base = g->h_off[b.first];
+        const int nitems = (int)(g->h_off[b.second] - base);
+        const int nseg = (int)(b.second - b.first);
+        if (nitems == 0) continue;
+        uint32_t *vals = g->d_adj + base;
+        hubkey_kernel<<<4096, 256>>>(vals, g->d_deg, (unsigned long long)nitems, kin);
+        rel_offsets_kernel<<<(nseg + 256) / 256, 256>>>(g->d_off, b.first, (uint32_t)nseg, rel);
+        CK(cudaGetLastError());
+        size_t tb = tb_max;
+        CK(cub::DeviceSegmentedSort::StableSortPairs(temp, tb, kin, kout, vals, vout, nitems, nseg, rel, rel + 1));
+        CK(cudaMemcpy(vals, vout, (size_t)nitems * 4, cudaMemcpyDeviceToDevice));
+      }
+      CK(cudaDeviceSynchronize());
+    } catch (...) {
+      for (void *p : tmp) cudaFree(p);
+      throw;
+    }
+    for (void *p : tmp) cudaFree(p);
+  });
+}
+
 extern "C" int ibfs_graph_info(const ibfs_graph *g, uint32_t *nv, uint64_t *ne, uint32_t *max_degree,
                                int *device) {
   return guarded([&] {
@@ -576,19 +633,42 @@ namespace {
 
 constexpr int LEVELS_PER_CHECK = 2;
 
-struct EventTimer {
-  std::vector<cudaEvent_t> ev;
-  size_t used = 0;
-  ~EventTimer() {
-    for (auto e : ev) cudaEventDestroy(e);
-  }
-  cudaEvent_t next() {
-    if (used == ev.size()) {
-      cudaEvent_t e;
-      CK(cudaEventCreate(&e));
-      ev.push_back(e);
+// Per-thread, per-device cache of CUDA events and a pinned host word buffer: creating
+// them per call (cudaEventCreate, cudaMallocHost) costs far more than a small level.
+struct DevCache {
+  std::vector<cudaEvent_t> timed, untimed;
+  void *pinned = nullptr;
+};
+struct ThreadCache {
+  std::vector<std::pair<int, DevCache>> devs;
+  ~ThreadCache() {
+    for (auto &d : devs) {
+      for (auto e : d.second.timed) cudaEventDestroy(e);
+      for (auto e : d.second.untimed) cudaEventDestroy(e);
+      if (d.second.pinned) cudaFreeHost(d.second.pinned);
     }
-    return ev[used++];
+  }
+  DevCache &get(int dev) {
+    for (auto &d : devs)
+      if (d.first == dev) return d.second;
+    devs.push_back({dev, DevCache{}});
+    return devs.back().second;
+  }
+};
+thread_local ThreadCache t_cache;
+
+struct EventTimer {
+  std::vector<cudaEvent_t> &pool;
+  bool timing;
+  size_t used = 0;
+  EventTimer(DevCache &dc, bool timed) : pool(timed ? dc.timed : dc.untimed), timing(timed) {}
+  cudaEvent_t next() {
+    if (used == pool.size()) {
+      cudaEvent_t e;
+      CK(cudaEventCreateWithFlags(&e, timing ? cudaEventDefault : cudaEventDisableTiming));
+      pool.push_back(e);
+    }
+    return pool[used++];
   }
 };
 
@@ -614,17 +694,26 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   const size_t rows_bytes_per_group = (size_t)W * nv;
   size_t free_b = 0, total_b = 0;
   CK(cudaMemGetInfo(&free_b, &total_b));
-  auto need = [&](uint32_t gg) {
-    return gg * (3 * gstride * B + (out_dev ? 0 : rows_bytes_per_group)) + (size_t)n * 24;
+  // memory: visited + R snapshot slots per group (+ device rows if the caller's buffer
+  // is not on the device); R >= 4, up to one slot per level when memory allows
+  auto need = [&](uint32_t gg, uint32_t r) {
+    return gg * ((1 + r) * gstride * B + 8 * (size_t)nv + (out_dev ? 0 : rows_bytes_per_group)) + (size_t)n * 24;
   };
-  while (G > 1 && need(G) > free_b / 10 * 8) G = (G + 1) / 2;
+  // The budget depends on the device size only (not on the momentary free memory), so
+  // repeated calls request identical scratch and the stream-ordered pool reuses it.
+  (void)free_b;
+  const size_t budget = total_b / 100 * 35;
+  while (G > 1 && need(G, 4) > budget) G = (G + 1) / 2;
+  uint32_t R = 4;
+  while (R < 24 && need(G, R + 1) <= budget) ++R;  // > R-2 levels: flushed ring rounds
 
   Scratch sc(g->device, stream);
   uint32_t *d_src = sc.get<uint32_t>(n);
   CK(cudaMemcpyAsync(d_src, sources, (size_t)n * 4, cudaMemcpyDefault, stream));
   T *visited = sc.get<T>(G * gstride);
-  T *buf0 = sc.get<T>(G * gstride);
-  T *buf1 = sc.get<T>(G * gstride);
+  T *ring = sc.get<T>((size_t)R * G * gstride);
+  uint32_t *tdq = sc.get<uint32_t>((size_t)G * nv);
+  uint32_t *buq = sc.get<uint32_t>((size_t)G * nv);
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
   LevelStat *lstat = sc.get<LevelStat>((size_t)G * MAXL);
   uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
@@ -634,8 +723,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   int8_t *staging = out_dev ? nullptr : sc.get<int8_t>((size_t)G * rows_bytes_per_group);
   CK(cudaMemsetAsync(flags, 0, 8, stream));
 
-  HostPinned pin(4096);
-  volatile uint32_t *h_done = (volatile uint32_t *)pin.p;  // [0..255] done slots, [256] range
+  DevCache &dc = t_cache.get(g->device);
+  if (!dc.pinned) CK(cudaMallocHost(&dc.pinned, 4096));
+  volatile uint32_t *h_done = (volatile uint32_t *)dc.pinned;  // [0..255] done slots, [256] range
   std::vector<LevelStat> h_lstat((size_t)G * MAXL);
   std::vector<unsigned long long> h_m((size_t)G * W), h_dig((size_t)G * W);
 
@@ -646,8 +736,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   a.nv = nv;
   a.gstride = gstride;
   a.visited = visited;
-  a.buf0 = buf0;
-  a.buf1 = buf1;
+  a.ring = ring;
+  a.R = (int)R;
+  a.gcap = (int)G;
   a.ctrl = ctrl;
   a.lstat = lstat;
   a.work_ctr = work_ctr;
@@ -656,13 +747,15 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   a.n_total = n;
   a.chunks = g->d_chunks;
   a.n_chunks = g->n_chunks;
-  a.tile_begin = g->d_tiles;
-  a.n_tiles = g->n_tiles;
+  a.tdq = tdq;
+  a.buq = buq;
+  a.n_iso = (uint32_t)(nv - g->nv_active);
   a.pol.mode = o.direction;
   a.pol.bu_from = o.bu_from;
   a.pol.alpha = o.alpha;
   a.pol.beta = o.beta;
   a.pol.nv_active = g->nv_active;
+  a.pol.ne = g->ne;
   a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
   for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
   uint32_t first_dir = 0;
@@ -670,17 +763,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   if (o.direction == IBFS_DIR_SCHEDULE && a.pol.sched_len > 0) first_dir = a.pol.sched[0];
 
   const int expand_grid = g->num_sms * g->expand_blocks_per_sm;
-  EventTimer timer;
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, kexp, kcom, kinit;
-  std::vector<cudaEvent_t> chk(256);
-  for (auto &e : chk) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-  struct EvGuard {
-    std::vector<cudaEvent_t> &v;
-    ~EvGuard() {
-      for (auto e : v) cudaEventDestroy(e);
-    }
-  } evg{chk};
-
+  EventTimer timer(dc, true), chk(dc, false);
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, kexp, kcom, kinit, kdep, kfin;
+  std::vector<int> klev;  // level of each timed expand/commit pair
   ibfs_stats st{};
   uint64_t launches = 0;
   bool range_error = false;
@@ -694,62 +779,83 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
     a.out = out_dev ? out_depths + (size_t)gb0 * rows_bytes_per_group : staging;
     const uint32_t rows_in_batch = std::min<uint32_t>(Gb * W, n - gb0 * W);
     CK(cudaMemsetAsync(flags, 0, 4, stream));
+    CK(cudaMemsetAsync(d_m, 0, (size_t)G * W * 8, stream));  // m_s accumulates in depth_kernel
     cudaEvent_t w0 = timer.next(), w1 = timer.next();
     CK(cudaEventRecord(w0, stream));
     {
       cudaEvent_t i0 = nullptr, i1 = nullptr;
       if (o.timing) { i0 = timer.next(); i1 = timer.next(); CK(cudaEventRecord(i0, stream)); }
       uint32_t bx = (uint32_t)std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, std::max<uint32_t>(1, 2048 / Gb));
-      init_state_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a);
+      init_ctrl_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
+      init_state_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a, first_dir);
       init_sources_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
       CK(cudaGetLastError());
-      launches += 2;
-      st.init_launches += 2;
-      st.init_bytes += (uint64_t)Gb * (3 * nv * B) + (uint64_t)rows_in_batch * nv;
+      launches += 3;
+      st.init_launches += 3;
+      st.init_bytes += (uint64_t)Gb * (3 * nv * B);
       if (o.timing) { CK(cudaEventRecord(i1, stream)); kinit.push_back({i0, i1}); }
     }
     const uint32_t commit_bx = (uint32_t)std::max<uint64_t>(
         1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, (uint64_t)g->num_sms * 8 / Gb));
+    // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
+    int flushed = -1;  // levels <= flushed are already in the rows
+    auto flush = [&](int l1) {
+      cudaEvent_t d0 = nullptr, d1 = nullptr;
+      if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
+      const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DT - 1) / DT,
+                                                                         (uint64_t)g->num_sms * 16 / Gb + 1));
+      depth_kernel<T><<<dim3(bx, Gb), DT, 0, stream>>>(a, flushed + 1, l1, flushed < 0 ? 1 : 0, d_m);
+      if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
+      launches++;
+      st.depth_launches++;
+      st.depth_bytes += (uint64_t)Gb * nv * (B * (uint64_t)(l1 - flushed)) + (uint64_t)rows_in_batch * nv;
+      flushed = l1;
+    };
     int level = 1;
     int chunk = 0;
-    int last_level_launched = 0;
+    cudaEvent_t chk_ev[256];
+    chk.used = 0;  // the previous batch's check events have completed
     while (level <= MAXL - 1) {
       const int lend = std::min(level + LEVELS_PER_CHECK, MAXL);
       for (int l = level; l < lend; ++l) {
+        // commit l zeroes slot (l+1) % R, which held level l+1-R: flush it first
+        if (l + 1 - (int)R > flushed) flush(l - 1);
         cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
         if (o.timing) { e0 = timer.next(); e1 = timer.next(); e2 = timer.next(); CK(cudaEventRecord(e0, stream)); }
-        expand_kernel<T><<<expand_grid, BLOCK, 0, stream>>>(a, l);
+        expand_kernel<T><<<expand_grid, BLOCK, sizeof(TileQueue<T>), stream>>>(a, l);
         if (o.timing) CK(cudaEventRecord(e1, stream));
         commit_kernel<T><<<dim3(commit_bx, Gb), BLOCK, 0, stream>>>(a, l);
-        if (o.timing) { CK(cudaEventRecord(e2, stream)); kexp.push_back({e0, e1}); kcom.push_back({e1, e2}); }
+        if (o.timing) {
+          CK(cudaEventRecord(e2, stream));
+          kexp.push_back({e0, e1});
+          kcom.push_back({e1, e2});
+          klev.push_back(l);
+        }
         launches += 2;
         st.expand_launches++;
         st.commit_launches++;
       }
       CK(cudaGetLastError());
-      last_level_launched = lend - 1;
       if (chunk >= 256) fail(IBFS_E_CUDA, "level loop overflow");
       CK(cudaMemcpyAsync((void *)(h_done + chunk), flags, 4, cudaMemcpyDeviceToHost, stream));
-      CK(cudaEventRecord(chk[chunk], stream));
+      cudaEvent_t ce = chk.next();
+      chk_ev[chunk] = ce;
+      CK(cudaEventRecord(ce, stream));
       ++chunk;
       level = lend;
       if (chunk >= 2) {
-        CK(cudaEventSynchronize(chk[chunk - 2]));
+        CK(cudaEventSynchronize(chk_ev[chunk - 2]));
         if (h_done[chunk - 2] >= Gb) break;
       }
     }
-    (void)last_level_launched;
+    flush(level - 1);  // the rest (each group stops at its own last level)
     CK(cudaEventRecord(w1, stream));
     win.push_back({w0, w1});
     // range check (a level-128 discovery means a depth > 127)
     CK(cudaMemcpyAsync((void *)(h_done + 256), flags + 1, 4, cudaMemcpyDeviceToHost, stream));
     // finalize: m_s and digests (outside the traversal window)
-    CK(cudaMemsetAsync(d_m, 0, (size_t)G * W * 8, stream));
-    {
-      uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, 2048 / Gb));
-      msum_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a, d_m);
-      launches++;
-    }
+    cudaEvent_t f0 = timer.next(), f1 = timer.next();
+    CK(cudaEventRecord(f0, stream));
     if (stats && stats->per_source_digest) {
       CK(cudaMemsetAsync(d_dig, 0, (size_t)G * W * 8, stream));
       uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, 64));
@@ -757,6 +863,8 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
       launches++;
     }
     CK(cudaGetLastError());
+    CK(cudaEventRecord(f1, stream));
+    kfin.push_back({f0, f1});
     CK(cudaMemcpyAsync(h_lstat.data(), lstat, (size_t)Gb * MAXL * sizeof(LevelStat), cudaMemcpyDeviceToHost, stream));
     CK(cudaMemcpyAsync(h_m.data(), d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
     if (stats && stats->per_source_digest)
@@ -793,8 +901,11 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
         P.new_pairs += L.newp;
         st.edges_inspected += L.insp;
         // DESIGN.md §5 byte model
-        uint64_t eb = (uint64_t)nv * B + 4 * L.jfq + 8 * L.proc + (4 + B) * L.insp + B * L.writes;
-        uint64_t cb = (uint64_t)nv * (3 * B + 4) + B * L.nf + L.newp;
+        // expand: per queued frontier its queue entry, row start, degree and word; per
+        // inspection the adjacency entry and the neighbour's word; per write one word.
+        // commit: S_l, visited and the zeroed slot streamed, visited written where new.
+        uint64_t eb = (16 + B) * L.proc + (4 + B) * L.insp + B * L.writes;
+        uint64_t cb = (uint64_t)nv * (3 * B + 4) + B * L.nf;
         st.expand_bytes += eb;
         st.commit_bytes += cb;
       }
@@ -803,12 +914,21 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   if (range_error) fail(IBFS_E_RANGE, "a depth exceeds 127 (int8 output)");
   // times
   for (auto &p : win) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.traverse_ms += ms; }
-  for (auto &p : kexp) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.expand_ms += ms; }
-  for (auto &p : kcom) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.commit_ms += ms; }
+  for (size_t i = 0; i < kexp.size(); ++i) {
+    float me = 0, mc = 0;
+    CK(cudaEventElapsedTime(&me, kexp[i].first, kexp[i].second));
+    CK(cudaEventElapsedTime(&mc, kcom[i].first, kcom[i].second));
+    st.expand_ms += me;
+    st.commit_ms += mc;
+    per_level[klev[i] - 1].expand_ms += me;
+    per_level[klev[i] - 1].commit_ms += mc;
+  }
   for (auto &p : kinit) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.init_ms += ms; }
+  for (auto &p : kfin) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.finalize_ms += ms; }
+  for (auto &p : kdep) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.depth_ms += ms; }
   st.n_groups = n_groups;
   st.n_launches = launches;
-  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes;
+  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes + st.depth_bytes;
   if (stats) {
     st.per_source_m = stats->per_source_m;
     st.per_source_digest = stats->per_source_digest;

@@ -3,23 +3,32 @@
 // One group = up to W BFS instances sharing one W-bit status word per vertex (the
 // Bitwise Status Array, §6).  Per group the device holds
 //   visited[v]  bit j = 1 iff instance j reached v at an earlier level  (BSA_k)
-//   buf0/buf1   alternate by level parity: F = discoveries of level l-1 (the top-down
-//               frontier words, Alg. 2 "BSA_k+1 XOR BSA_k" P:L793), N = discoveries of
-//               level l being accumulated (the new bits of BSA_k+1, Alg. 1).
+//   S_l[v]      ring of R level snapshots (slot l % R): the bits discovered at level l,
+//               i.e. BSA_l+1 XOR BSA_l.  S_l-1 is the top-down frontier word F of level
+//               l (Alg. 2 "BSA_k+1 XOR BSA_k"); S_l accumulates level l's new bits
+//               (Alg. 1).  S_0 holds the sources.
+//   tdq / buq   the joint frontier queues (JFQ) of the next level, one per
+//               direction, written by the commit that precedes it: top-down = vertices
+//               with new bits (Alg. 2 l.3 "BSA_k+1 XOR BSA_k"), bottom-up = vertices with
+//               an unvisited active bit (Alg. 2 l.7, reading #6).  Each array holds
+//               "light" vertices (degree <= LIGHT_DEG) from the front and "heavy" ones
+//               from the back; a shared frontier is enqueued once.
 // Level l (discovers depth l; reading #20) is two launches:
-//   expand_kernel<T>(l): builds the joint frontier queue per vertex tile with a warp
-//       ballot (Alg. 2; JFQ P:L329-L335) and expands it --
+//   expand_kernel<T>(l): expands the level's JFQ --
 //       top-down  N[w] |= F[f] & ~visited[w]   with RED.OR (Alg. 1 l.5),
 //       bottom-up acc  |= visited[w] & T[f], T = ~visited[f] & active, early exit when
 //                 acc == T (Alg. 1 l.7-10; reading #5), N[f] = acc.
-//   commit_kernel<T>(l): visited |= N, depth[j][v] = l for every new bit j (P:L779
-//       "the differences between BSA_k and BSA_k+1 are used to identify the just visited
-//       vertices"), clears the old frontier buffer, counts the direction-switch inputs,
-//       and its last CTA per group decides the next level's direction (reading #7).
-// Work decomposition (static, built at load): edge-balanced vertex tiles of at most
-// V_TILE vertices / E_TILE non-hub edges, plus hub chunks of CHUNK edges for vertices of
-// degree > HUB_T (the paper's shared-memory "cache" of a frontier's adjacency shared by
-// all instances, becomes a CTA-cooperative expansion of the hub's row).
+//   commit_kernel<T>(l): visited |= S_l ("the differences between BSA_k and
+//       BSA_k+1 are used to identify the just visited vertices"), zeroes slot l+1, builds
+//       both queues of level l+1 with warp ballots (the paper's __any/__ballot JFQ
+//       generation), counts the direction-switch inputs; its last CTA per group
+//       decides the next level's direction (reading #7).
+//   depth_kernel<T>: depth[j][v] = the level l whose snapshot first holds bit j of v
+//       (-1 if none), written row-major through a shared-memory transpose, once per
+//       ring round (normally once per group, after the last level); also sums m_s.
+// Vertices of degree > HUB_T never enter the queues: their rows are split into static
+// chunks of CHUNK edges that whole CTAs sweep (the paper's shared "cache" of a
+// frontier's adjacency used by all instances, as CTA-cooperative expansion).
 #pragma once
 #include <cstdint>
 #include "word.cuh"
@@ -28,14 +37,21 @@ namespace ibfs {
 
 constexpr int BLOCK = 256;
 constexpr int NWARP = BLOCK / 32;
-constexpr int V_TILE = 1024;
-constexpr int E_TILE = 8192;
-constexpr int HUB_T = 8192;
-constexpr int CHUNK = 8192;
-constexpr int BU_WARP_DEG = 32;
-constexpr int MAXL = 130;       // level index 1..129 (129 only detects depth > 127)
-constexpr int MAX_G = 64;       // groups per launch batch
+constexpr int QL = 1024;         // light-queue entries per work item
+constexpr int QH = 32;           // heavy TD-queue entries per work item
+constexpr int QBH = 256;         // heavy BU-queue entries per work item
+constexpr int LIGHT_DEG = 32;    // degree <= LIGHT_DEG: light
+constexpr int HUB_T = 8192;      // degree > HUB_T: hub (chunked rows)
+constexpr int CHUNK = 8192;      // hub-row edges per work item
+constexpr int MAXL = 130;        // level index 1..129 (129 only detects depth > 127)
+constexpr int MAX_G = 64;        // groups per launch batch
 constexpr unsigned FULL = 0xffffffffu;
+#ifndef IBFS_EXPAND_MINB
+#define IBFS_EXPAND_MINB 3  // min resident expand CTAs per SM (register cap)
+#endif
+
+// queue classes
+constexpr int Q_TDL = 0, Q_TDH = 1, Q_BUL = 2, Q_BUH = 3;
 
 struct HubChunk {
   unsigned long long e0, e1;
@@ -53,11 +69,13 @@ template <typename T>
 struct GroupCtrl {
   T active;   // instances that discovered something at the last committed level
   T newacc;   // OR of the new bits of the running commit
-  unsigned long long n_f, m_f, m_u, newp;
-  uint32_t dir;     // direction of the next expand: 0 TD, 1 BU
+  unsigned long long n_f, m_f, newp;
+  uint32_t qlen[2][4];  // [parity of the producing level][queue class]
+  uint32_t dir;         // direction of the next expand: 0 TD, 1 BU
   uint32_t done;
   uint32_t arrive;
   uint32_t last_level;
+  uint32_t iso_jfq1, iso_fq1;  // isolated-vertex part of a bottom-up level 1 (stats)
 };
 
 struct Policy {
@@ -65,6 +83,7 @@ struct Policy {
   uint32_t bu_from;
   float alpha, beta;
   unsigned long long nv_active;  // vertices with degree > 0
+  unsigned long long ne;         // CSR entries
   uint32_t sched_len;
   uint8_t sched[MAXL];  // 0 TD / 1 BU for level l at index l-1
 };
@@ -76,7 +95,11 @@ struct BatchArgs {
   const uint32_t *deg;
   uint32_t nv;
   size_t gstride;  // words per per-group array
-  T *visited, *buf0, *buf1;
+  T *visited;
+  T *ring;       // [R][gcap][gstride] level snapshots
+  int R;         // ring slots
+  int gcap;      // groups allocated per slot
+  uint32_t *tdq, *buq;  // [gcap][nv] queues
   GroupCtrl<T> *ctrl;
   LevelStat *lstat;     // [G][MAXL]
   uint32_t *work_ctr;   // [MAXL]
@@ -89,8 +112,7 @@ struct BatchArgs {
   int8_t *out;          // row g*W + j of this batch at out + (g*W + j) * nv
   const HubChunk *chunks;
   uint32_t n_chunks;
-  const uint32_t *tile_begin;  // [n_tiles + 1]
-  uint32_t n_tiles;
+  uint32_t n_iso;       // vertices of degree 0
   Policy pol;
 };
 
@@ -102,12 +124,25 @@ __device__ __forceinline__ int group_rows(const BatchArgs<T> &a, int g) {
 }
 
 template <typename T>
+__device__ __forceinline__ T *snap(const BatchArgs<T> &a, int g, int level) {
+  return a.ring + ((size_t)(level % a.R) * a.gcap + g) * a.gstride;
+}
+template <typename T>
 __device__ __forceinline__ T *frontier_buf(const BatchArgs<T> &a, int g, int level) {
-  return ((level - 1) & 1 ? a.buf1 : a.buf0) + (size_t)g * a.gstride;
+  return snap(a, g, level - 1);
 }
 template <typename T>
 __device__ __forceinline__ T *next_buf(const BatchArgs<T> &a, int g, int level) {
-  return (level & 1 ? a.buf1 : a.buf0) + (size_t)g * a.gstride;
+  return snap(a, g, level);
+}
+template <typename T>
+__device__ __forceinline__ uint32_t *queue_of(const BatchArgs<T> &a, int g, int cls) {
+  return (cls < Q_BUL ? a.tdq : a.buq) + (size_t)g * a.nv;
+}
+// entry i of queue class cls (light classes from the front, heavy from the back)
+template <typename T>
+__device__ __forceinline__ uint32_t queue_at(const BatchArgs<T> &a, const uint32_t *q, int cls, uint32_t i) {
+  return (cls & 1) ? q[a.nv - 1 - i] : q[i];
 }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -116,88 +151,160 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return m;
 }
 
-// ------------------------------------------------------------------------- init ----
-// Zero the group's status arrays and fill its depth rows with -1 (a2).
+// Warp-aggregated append of this lane's vertex v to queue class cls when pred holds
+// (one atomic per warp per class, "__ballot()").
 template <typename T>
-__global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a) {
-  constexpr int W = WordBits<T>::value;
-  const int g = blockIdx.y;
-  const size_t stride = (size_t)gridDim.x * BLOCK;
-  const T z = wzero_value<T>();
-  T *vis = a.visited + (size_t)g * a.gstride;
-  T *b0 = a.buf0 + (size_t)g * a.gstride;
-  T *b1 = a.buf1 + (size_t)g * a.gstride;
-  for (size_t v = (size_t)blockIdx.x * BLOCK + threadIdx.x; v < a.nv; v += stride) {
-    st(vis + v, z);
-    st(b0 + v, z);
-    st(b1 + v, z);
+__device__ __forceinline__ void queue_push(const BatchArgs<T> &a, int g, uint32_t *qlen, int cls,
+                                           bool pred, uint32_t v) {
+  const uint32_t bal = __ballot_sync(FULL, pred);
+  if (!bal) return;
+  const int lane = threadIdx.x & 31;
+  const int leader = __ffs(bal) - 1;
+  uint32_t base = 0;
+  if (lane == leader) base = atomicAdd(qlen + cls, (uint32_t)__popc(bal));
+  base = __shfl_sync(FULL, base, leader);
+  if (pred) {
+    const uint32_t i = base + __popc(bal & lanemask_lt());
+    uint32_t *q = queue_of(a, g, cls);
+    if (cls & 1) q[a.nv - 1 - i] = v; else q[i] = v;
   }
-  const int rows = group_rows(a, g);
-  if (rows == 0) return;
-  int8_t *base = a.out + (size_t)g * W * a.nv;
-  const size_t bytes = (size_t)rows * a.nv;
-  // head bytes up to 16-byte alignment, then 16-byte stores, then the tail
-  size_t head = (16 - ((uintptr_t)base & 15)) & 15;
-  if (head > bytes) head = bytes;
-  const size_t gid = (size_t)blockIdx.x * BLOCK + threadIdx.x;
-  if (gid < head) base[gid] = -1;
-  const size_t nvec = (bytes - head) / 16;
-  int4 *vp = reinterpret_cast<int4 *>(base + head);
-  const int4 m1 = make_int4(-1, -1, -1, -1);
-  for (size_t i = gid; i < nvec; i += stride) vp[i] = m1;
-  const size_t tail0 = head + nvec * 16;
-  if (gid < bytes - tail0) base[tail0 + gid] = -1;
 }
 
-// Sources: visited[s_j] |= bit j, F[s_j] |= bit j, depth[j][s_j] = 0; control words.
+__device__ __forceinline__ int queue_class(uint32_t d, bool bu) {
+  return (bu ? Q_BUL : Q_TDL) + (d > (uint32_t)LIGHT_DEG ? 1 : 0);
+}
+
+// ------------------------------------------------------------------------- init ----
+// Control words, per-level counters and the item counters (one CTA per group).
 template <typename T>
-__global__ void init_sources_kernel(BatchArgs<T> a, uint32_t first_dir) {
-  constexpr int W = WordBits<T>::value;
+__global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
   const int g = blockIdx.x;
   const int rows = group_rows(a, g);
-  T *vis = a.visited + (size_t)g * a.gstride;
-  T *f = a.buf0 + (size_t)g * a.gstride;  // frontier buffer of level 1
-  for (int j = threadIdx.x; j < rows; j += blockDim.x) {
-    uint32_t s = a.src[(size_t)g * W + j];
-    set_bit_atomic(vis + s, j);
-    set_bit_atomic(f + s, j);
-    a.out[((size_t)g * W + j) * a.nv + s] = 0;
-  }
   LevelStat *ls = a.lstat + (size_t)g * MAXL;
   for (int l = threadIdx.x; l < MAXL; l += blockDim.x) ls[l] = LevelStat{};
   if (threadIdx.x == 0) {
     GroupCtrl<T> c;
     c.active = wlowmask<T>(rows);
     c.newacc = wzero_value<T>();
-    c.n_f = c.m_f = c.m_u = c.newp = 0;
+    c.n_f = c.m_f = c.newp = 0;
+    for (int p = 0; p < 2; ++p)
+      for (int k = 0; k < 4; ++k) c.qlen[p][k] = 0;
     c.dir = first_dir;
     c.done = rows == 0 ? 1u : 0u;
     c.arrive = 0;
     c.last_level = 0;
+    c.iso_jfq1 = c.iso_fq1 = 0;
     a.ctrl[g] = c;
     if (rows == 0) atomicAdd(a.batch_done, 1u);
   }
-  if (g == 0) {
+  if (g == 0)
     for (int l = threadIdx.x; l < MAXL; l += blockDim.x) a.work_ctr[l] = 0;
+}
+
+// Zero the group's visited words and the snapshot slots of levels 0 and 1 (a2); when
+// level 1 runs bottom-up, enqueue every vertex of degree 1..HUB_T (all are unvisited
+// for some instance unless they are the source of every instance -- the expand skips
+// those).
+template <typename T>
+__global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint32_t first_dir) {
+  const int g = blockIdx.y;
+  if (group_rows(a, g) == 0) return;
+  const size_t stride = (size_t)gridDim.x * BLOCK;
+  const T z = wzero_value<T>();
+  T *vis = a.visited + (size_t)g * a.gstride;
+  T *s0 = snap(a, g, 0);
+  T *s1 = snap(a, g, 1);
+  uint32_t *qlen = a.ctrl[g].qlen[0];
+  const size_t nvr = ((size_t)a.nv + 31) & ~(size_t)31;  // warp-uniform trip count
+  for (size_t v = (size_t)blockIdx.x * BLOCK + threadIdx.x; v < nvr; v += stride) {
+    const bool in = v < a.nv;
+    if (in) {
+      st(vis + v, z);
+      st(s0 + v, z);
+      st(s1 + v, z);
+    }
+    if (first_dir) {
+      const uint32_t d = in ? __ldg(a.deg + v) : 0u;
+      const bool q = d > 0 && d <= (uint32_t)HUB_T;
+      queue_push(a, g, qlen, Q_BUL, q && d <= (uint32_t)LIGHT_DEG, (uint32_t)v);
+      queue_push(a, g, qlen, Q_BUH, q && d > (uint32_t)LIGHT_DEG, (uint32_t)v);
+    }
+  }
+}
+
+// Sources: visited[s_j] |= bit j, S_0[s_j] |= bit j (depth 0); the distinct non-hub
+// source vertices form the top-down queue of level 1; level-1 statistics.
+template <typename T>
+__global__ void init_sources_kernel(BatchArgs<T> a, uint32_t first_dir) {
+  constexpr int W = WordBits<T>::value;
+  __shared__ uint32_t s_src[W];
+  __shared__ uint32_t s_cnt[3];
+  const int g = blockIdx.x;
+  const int rows = group_rows(a, g);
+  if (rows == 0) return;
+  T *vis = a.visited + (size_t)g * a.gstride;
+  T *f = snap(a, g, 0);  // frontier of level 1
+  if (threadIdx.x < 3) s_cnt[threadIdx.x] = 0;
+  for (int j = threadIdx.x; j < rows; j += blockDim.x) s_src[j] = a.src[(size_t)g * W + j];
+  __syncthreads();
+  uint32_t *qlen = a.ctrl[g].qlen[0];
+  for (int j = threadIdx.x; j < W; j += blockDim.x) {  // warp-uniform loop
+    bool first = false;
+    uint32_t s = 0, d = 0;
+    if (j < rows) {
+      s = s_src[j];
+      set_bit_atomic(vis + s, j);
+      set_bit_atomic(f + s, j);
+      first = true;
+      for (int i = 0; i < j; ++i)
+        if (s_src[i] == s) { first = false; break; }
+      d = __ldg(a.deg + s);
+      if (first) atomicAdd(&s_cnt[0], 1u);          // distinct sources: |JFQ| of level 1
+      if (d == 0) atomicAdd(&s_cnt[1], 1u);         // rows whose source is isolated
+    }
+    const bool q = first && d > 0 && d <= (uint32_t)HUB_T && first_dir == 0;
+    queue_push(a, g, qlen, Q_TDL, q && d <= (uint32_t)LIGHT_DEG, s);
+    queue_push(a, g, qlen, Q_TDH, q && d > (uint32_t)LIGHT_DEG, s);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    LevelStat *ls = a.lstat + (size_t)g * MAXL + 1;
+    if (first_dir == 0) {
+      ls->jfq = s_cnt[0];
+      ls->fq = (unsigned long long)rows;
+    } else {
+      // bottom-up level 1, isolated vertices: T = active & ~(own source bits)
+      bool all_same_iso = __ldg(a.deg + s_src[0]) == 0;
+      for (int j = 1; j < rows && all_same_iso; ++j) all_same_iso = s_src[j] == s_src[0];
+      ls->jfq = (unsigned long long)a.n_iso - (all_same_iso ? 1u : 0u);
+      ls->fq = (unsigned long long)a.n_iso * rows - s_cnt[1];
+    }
   }
 }
 
 // ----------------------------------------------------------------------- expand ----
-struct ExpandSmem {
-  unsigned long long start[V_TILE];
-  uint32_t aux[V_TILE + 1];  // TD: degree prefix; BU: degree
-  uint32_t vtx[V_TILE];
+struct ExpandSmem {  // static part
   uint32_t wsum[NWARP];
   uint32_t cnt[2];
   uint32_t item;
   uint32_t flag;
+  uint32_t nitems[3][MAX_G + 1];     // per class group (heavy / light) item prefix
   unsigned long long acc[MAX_G][5];  // jfq, fq, proc, insp, writes
 };
 
-// Exclusive scan of s[0..n) in place (n <= V_TILE), s[n] = total.  Block-wide.
+// Dynamic part: the CTA-local copy of one work item's queue entries.
+template <typename T>
+struct TileQueue {
+  unsigned long long start[QL];  // adjacency row start of entry i
+  T word[QL];                    // TD: frontier word F; BU: target T
+  uint32_t aux[QL + 1];          // degrees, then their exclusive prefix
+  uint32_t vtx[QL];
+};
+
+// Exclusive scan of s[0..n) in place (n <= QL), s[n] = total.  Block-wide.
 __device__ __forceinline__ void block_exclusive_scan(uint32_t *s, uint32_t n, uint32_t *wsum) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  constexpr int PER = V_TILE / BLOCK;  // 4 consecutive entries per thread
+  constexpr int PER = QL / BLOCK;  // 4 consecutive entries per thread
   uint32_t x[PER];
   uint32_t sum = 0;
 #pragma unroll
@@ -236,7 +343,7 @@ __device__ __forceinline__ void block_exclusive_scan(uint32_t *s, uint32_t n, ui
   __syncthreads();
 }
 
-// Largest q in [0, n) with s[q] <= e (s strictly increasing, s[0] = 0, s[n] > e).
+// Largest q in [0, n) with s[q] <= e (s strictly increasing on the queued entries).
 __device__ __forceinline__ uint32_t lbs_search(const uint32_t *s, uint32_t n, uint32_t e) {
   uint32_t lo = 0, hi = n;
   while (hi - lo > 1) {
@@ -246,7 +353,6 @@ __device__ __forceinline__ uint32_t lbs_search(const uint32_t *s, uint32_t n, ui
   return lo;
 }
 
-template <typename T>
 __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq, uint32_t fq,
                                              uint32_t proc, uint32_t insp, uint32_t writes) {
   jfq = __reduce_add_sync(FULL, jfq);
@@ -263,46 +369,29 @@ __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq
   }
 }
 
-// Top-down tile: ballot-compact the frontiers (F != 0) of the tile into a CTA-local
-// JFQ, then an edge-balanced sweep over their rows (load-balanced search on the degree
-// prefix), OR-ing the frontier word into each unvisited neighbour (Alg. 1 l.4-5).
+// Top-down item: entries [i0, i1) of a TD queue class.  The frontier words and rows of
+// the entries are staged in shared memory, then an edge-balanced sweep (load-balanced
+// search on the degree prefix) ORs each frontier word into its unvisited neighbours
+// (Alg. 1 l.4-5): consecutive threads read consecutive adjacency entries.
 template <typename T>
-__device__ void tile_td(const BatchArgs<T> &a, ExpandSmem &sm, T *s_word, int g, uint32_t t,
-                        int level) {
-  const int tid = threadIdx.x, lane = tid & 31;
-  const uint32_t vb = a.tile_begin[t], ve = a.tile_begin[t + 1];
+__device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq, int g, int cls,
+                        uint32_t i0, uint32_t i1, int level) {
+  const int tid = threadIdx.x;
   const T *F = frontier_buf(a, g, level);
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
-  uint32_t jfq = 0, fq = 0, insp = 0, writes = 0;
-  if (tid == 0) sm.cnt[0] = 0;
-  __syncthreads();
-  for (uint32_t base = vb; base < ve; base += BLOCK) {
-    const uint32_t v = base + tid;
-    const bool in = v < ve;
-    T f = in ? ldg(F + v) : wzero_value<T>();
-    const bool nz = !wzero(f);
-    uint32_t d = nz ? __ldg(a.deg + v) : 0u;
-    const bool isq = nz && d <= (uint32_t)HUB_T;
-    if (isq) { jfq++; fq += wpopc(f); }
-    const bool keep = isq && d > 0;
-    const uint32_t bal = __ballot_sync(FULL, keep);
-    if (bal) {
-      uint32_t wb = 0;
-      if (lane == 0) wb = atomicAdd(&sm.cnt[0], (uint32_t)__popc(bal));
-      wb = __shfl_sync(FULL, wb, 0);
-      if (keep) {
-        const uint32_t pos = wb + __popc(bal & lanemask_lt());
-        sm.start[pos] = __ldg(a.off + v);
-        s_word[pos] = f;
-        sm.aux[pos] = d;
-      }
-    }
+  const uint32_t *q = queue_of(a, g, cls);
+  const uint32_t qn = i1 - i0;
+  uint32_t insp = 0, writes = 0;
+  for (uint32_t i = tid; i < qn; i += BLOCK) {
+    const uint32_t v = queue_at(a, q, cls, i0 + i);
+    tq.start[i] = __ldg(a.off + v);
+    tq.word[i] = ldg(F + v);
+    tq.aux[i] = __ldg(a.deg + v);
   }
   __syncthreads();
-  const uint32_t qn = sm.cnt[0];
-  block_exclusive_scan(sm.aux, qn, sm.wsum);
-  const uint32_t total = sm.aux[qn];
+  block_exclusive_scan(tq.aux, qn, sm.wsum);
+  const uint32_t total = tq.aux[qn];
   constexpr int U = 4;
   for (uint32_t e0 = 0; e0 < total; e0 += BLOCK * U) {
     uint32_t w[U];
@@ -312,9 +401,9 @@ __device__ void tile_td(const BatchArgs<T> &a, ExpandSmem &sm, T *s_word, int g,
       const uint32_t e = e0 + u * BLOCK + tid;
       w[u] = 0xffffffffu;
       if (e < total) {
-        const uint32_t q = lbs_search(sm.aux, qn, e);
-        w[u] = __ldg(a.adj + sm.start[q] + (e - sm.aux[q]));
-        fw[u] = s_word[q];
+        const uint32_t k = lbs_search(tq.aux, qn, e);
+        w[u] = __ldg(a.adj + tq.start[k] + (e - tq.aux[k]));
+        fw[u] = tq.word[k];
       }
     }
 #pragma unroll
@@ -326,94 +415,131 @@ __device__ void tile_td(const BatchArgs<T> &a, ExpandSmem &sm, T *s_word, int g,
       }
     }
   }
-  flush_counts<T>(sm, g, jfq, fq, qn > 0 && tid == 0 ? qn : 0u, insp, writes);
+  flush_counts(sm, g, 0u, 0u, tid == 0 ? qn : 0u, insp, writes);
 }
 
-// Bottom-up tile: every vertex with an unvisited active bit (T = ~visited & active) is a
-// frontier (Alg. 2 l.7, reading #6); it ORs its neighbours' visited words masked by T,
-// in CSR order, and stops as soon as the accumulated word covers T (early termination,
-// P:L817 with the active mask of reading #5).  Degree <= 32: one thread per vertex;
-// larger: one warp per vertex with a warp OR-reduce and a warp-wide exit test.
+// Bottom-up item: entries [i0, i1) of a BU queue class.
+// Every entry f with T = active & ~visited[f] != 0 is a frontier (Alg. 2 l.7, reading
+// #6); it ORs its neighbours' visited words masked by T in CSR order and stops once the
+// accumulated word covers T (early termination, active mask of reading #5).  One
+// thread owns one frontier at a time ("a single thread to work on each frontier",
+// P:L813) and inspects 4 neighbours per step, with the next step's adjacency loads in
+// flight during this step's gathers; each warp refills its lanes from a private ring as
+// soon as a frontier terminates, so lanes stay busy until the item drains.
 template <typename T>
-__device__ void tile_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_word, int g, uint32_t t,
-                        int level, T active) {
+struct BuRing {  // per-warp rings of QL / NWARP entries, carved from TileQueue storage
+  unsigned long long start[QL];
+  T word[QL];
+  uint32_t deg[QL];
+  uint32_t vtx[QL];
+};
+
+template <typename T>
+__device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq, int g, int cls,
+                        uint32_t i0, uint32_t i1, int level, T active) {
+  constexpr int QW = QL / NWARP;  // ring entries per warp (128)
+  static_assert(sizeof(BuRing<T>) <= sizeof(TileQueue<T>), "BU ring must fit the item storage");
+  BuRing<T> &bq = *reinterpret_cast<BuRing<T> *>(&tq);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t vb = a.tile_begin[t], ve = a.tile_begin[t + 1];
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
+  const uint32_t *q = queue_of(a, g, cls);
   uint32_t jfq = 0, fq = 0, proc = 0, insp = 0, writes = 0;
-  if (tid == 0) { sm.cnt[0] = 0; sm.cnt[1] = 0; }
+  if (tid == 0) sm.cnt[0] = i0;
   __syncthreads();
-  for (uint32_t base = vb; base < ve; base += BLOCK) {
-    const uint32_t v = base + tid;
-    const bool in = v < ve;
-    T tg = wzero_value<T>();
-    if (in) tg = wandn(active, ldg(vis + v));
-    const bool nz = !wzero(tg);
-    const uint32_t d = nz ? __ldg(a.deg + v) : 0u;
-    const bool isq = nz && d <= (uint32_t)HUB_T;
-    if (isq) { jfq++; fq += wpopc(tg); }
-    const bool small = isq && d > 0 && d <= (uint32_t)BU_WARP_DEG;
-    const bool large = isq && d > (uint32_t)BU_WARP_DEG;
-    const uint32_t bs = __ballot_sync(FULL, small);
-    const uint32_t bl = __ballot_sync(FULL, large);
-    uint32_t ws = 0, wl = 0;
-    if (lane == 0) {
-      if (bs) ws = atomicAdd(&sm.cnt[0], (uint32_t)__popc(bs));
-      if (bl) wl = atomicAdd(&sm.cnt[1], (uint32_t)__popc(bl));
+  const int qbase = warp * QW;
+  uint32_t head = 0, tail = 0;  // warp-uniform ring cursors
+  bool range_done = false;
+  bool has = false;
+  uint32_t v = 0, d = 0, k = 0;
+  unsigned long long s0 = 0;
+  T tg = wzero_value<T>(), acc = wzero_value<T>();
+  uint32_t wn[4];  // adjacency entries of the lane's next step (prefetched)
+  // refill pipeline: the loads for the next 32 queue entries are issued one round early
+  uint32_t c_next = 0, x_next = 0, dx_next = 0;
+  T tx_next = wzero_value<T>();
+  unsigned long long ox_next = 0;
+  auto issue_refill = [&]() {
+    if (lane == 0) c_next = atomicAdd(&sm.cnt[0], 32u);
+    c_next = __shfl_sync(FULL, c_next, 0);
+    const uint32_t i = c_next + lane;
+    if (c_next < i1 && i < i1) {
+      x_next = queue_at(a, q, cls, i);
+      tx_next = wandn(active, ldg(vis + x_next));
+      dx_next = __ldg(a.deg + x_next);
+      ox_next = __ldg(a.off + x_next);
+    } else {
+      tx_next = wzero_value<T>();
+      dx_next = 0;
     }
-    ws = __shfl_sync(FULL, ws, 0);
-    wl = __shfl_sync(FULL, wl, 0);
-    if (small || large) {
-      const uint32_t pos = small ? ws + __popc(bs & lanemask_lt())
-                                 : (uint32_t)(V_TILE - 1) - (wl + __popc(bl & lanemask_lt()));
-      sm.start[pos] = __ldg(a.off + v);
-      s_word[pos] = tg;
-      sm.aux[pos] = d;
-      sm.vtx[pos] = v;
+  };
+  issue_refill();
+  for (;;) {
+    if (!range_done && tail - head <= (uint32_t)(QW - 32)) {
+      if (c_next >= i1) {
+        range_done = true;
+      } else {
+        const T tx = tx_next;
+        const bool keep = !wzero(tx);
+        if (keep) { jfq++; fq += wpopc(tx); }
+        const uint32_t bal = __ballot_sync(FULL, keep);
+        if (keep) {
+          const uint32_t pos = qbase + ((tail + __popc(bal & lanemask_lt())) & (QW - 1));
+          bq.start[pos] = ox_next;
+          bq.word[pos] = tx;
+          bq.deg[pos] = dx_next;
+          bq.vtx[pos] = x_next;
+        }
+        tail += __popc(bal);
+        __syncwarp();
+        issue_refill();
+      }
     }
-  }
-  __syncthreads();
-  const uint32_t ns = sm.cnt[0], nl = sm.cnt[1];
-  // thread per low-degree vertex
-  for (uint32_t q = tid; q < ns; q += BLOCK) {
-    const unsigned long long s0 = sm.start[q];
-    const uint32_t d = sm.aux[q];
-    const T tg = s_word[q];
-    T acc = wzero_value<T>();
-    proc++;
-    for (uint32_t k = 0; k < d; k += 4) {
+    const uint32_t idle = __ballot_sync(FULL, !has);
+    const uint32_t avail = tail - head;
+    if (!has) {
+      const uint32_t r = __popc(idle & lanemask_lt());
+      if (r < avail) {
+        const uint32_t pos = qbase + ((head + r) & (QW - 1));
+        s0 = bq.start[pos];
+        tg = bq.word[pos];
+        d = bq.deg[pos];
+        v = bq.vtx[pos];
+        k = 0;
+        acc = wzero_value<T>();
+        has = true;
+        proc++;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) wn[u] = ((uint32_t)u < d) ? __ldg(a.adj + s0 + u) : 0xffffffffu;
+      }
+    }
+    head += min((uint32_t)__popc(idle), avail);
+    __syncwarp();
+    const uint32_t busy = __ballot_sync(FULL, has);
+    if (!busy) {
+      if (range_done && head == tail) break;
+      continue;
+    }
+    if (has) {
       uint32_t w[4];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) w[u] = (k + u < d) ? __ldg(a.adj + s0 + k + u) : 0xffffffffu;
+      for (int u = 0; u < 4; ++u) w[u] = wn[u];
+      T x[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) x[u] = w[u] != 0xffffffffu ? ldg(vis + w[u]) : wzero_value<T>();
+      k += 4;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) wn[u] = (k + u < d) ? __ldg(a.adj + s0 + k + u) : 0xffffffffu;
 #pragma unroll
       for (int u = 0; u < 4; ++u)
-        if (w[u] != 0xffffffffu) { acc = wor(acc, wand(ldg(vis + w[u]), tg)); insp++; }
-      if (weq(acc, tg)) break;
-    }
-    if (!wzero(acc)) { st(N + sm.vtx[q], acc); writes++; }
-  }
-  // warp per higher-degree vertex
-  for (uint32_t q = warp; q < nl; q += NWARP) {
-    const uint32_t idx = V_TILE - 1 - q;
-    const unsigned long long s0 = sm.start[idx];
-    const uint32_t d = sm.aux[idx];
-    const T tg = s_word[idx];
-    T acc = wzero_value<T>();
-    if (lane == 0) proc++;
-    for (uint32_t k = 0; k < d; k += 32) {
-      T x = wzero_value<T>();
-      if (k + lane < d) {
-        const uint32_t w = __ldg(a.adj + s0 + k + lane);
-        x = wand(ldg(vis + w), tg);
-        insp++;
+        if (w[u] != 0xffffffffu) { acc = wor(acc, wand(x[u], tg)); insp++; }
+      if (weq(acc, tg) || k >= d) {
+        if (!wzero(acc)) { st(N + v, acc); writes++; }
+        has = false;
       }
-      acc = wor(acc, warp_or(x));
-      if (weq(acc, tg)) break;
     }
-    if (lane == 0 && !wzero(acc)) { st(N + sm.vtx[idx], acc); writes++; }
   }
-  flush_counts<T>(sm, g, jfq, fq, proc, insp, writes);
+  flush_counts(sm, g, jfq, fq, proc, insp, writes);
 }
 
 // Hub chunk, top-down: CHUNK edges of one hub's row swept by the whole CTA.
@@ -426,7 +552,7 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
   const T f = ldg(F + c.v);
   if (wzero(f)) return;
   uint32_t insp = 0, writes = 0;
-  constexpr int U = 4;
+  constexpr int U = 8;
   for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
     uint32_t w[U];
 #pragma unroll
@@ -444,8 +570,7 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
     }
   }
   const bool first = c.first && tid == 0;
-  flush_counts<T>(sm, g, first ? 1u : 0u, first ? (uint32_t)wpopc(f) : 0u, first ? 1u : 0u, insp,
-                  writes);
+  flush_counts(sm, g, 0u, 0u, first ? 1u : 0u, insp, writes);
 }
 
 // Hub chunk, bottom-up: the CTA ORs a chunk of the hub's neighbours in waves, with a
@@ -488,43 +613,75 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
     }
     if (tid == 0 && !wzero(acc)) { red_or(N + c.v, acc); writes++; }
   }
-  flush_counts<T>(sm, g, first ? 1u : 0u, first ? (uint32_t)wpopc(tg) : 0u, first ? 1u : 0u, insp,
-                  writes);
+  flush_counts(sm, g, first ? 1u : 0u, first ? (uint32_t)wpopc(tg) : 0u, first ? 1u : 0u, insp, writes);
 }
 
-// One launch per level for all groups of a batch.  CTAs pull work items (hub chunks
-// first, then tiles) from a per-level counter; each item carries its group, whose
-// direction for this level was decided by the previous commit.
+// One launch per level for all groups of a batch.  Work items, pulled by CTAs from a
+// per-level counter: all hub chunks first, then heavy-queue items, then light-queue
+// items, each carrying its group (whose direction the previous commit decided).
 template <typename T>
-__global__ void __launch_bounds__(BLOCK) expand_kernel(BatchArgs<T> a, int level) {
+__global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) expand_kernel(BatchArgs<T> a, int level) {
   __shared__ ExpandSmem sm;
-  __shared__ T s_word[V_TILE];
   __shared__ T s_red[NWARP];
+  extern __shared__ __align__(16) unsigned char dyn_smem[];
+  TileQueue<T> &tq = *reinterpret_cast<TileQueue<T> *>(dyn_smem);
   const int tid = threadIdx.x;
   if (*(volatile uint32_t *)a.batch_done >= (uint32_t)a.G) return;
   for (int i = tid; i < a.G * 5; i += BLOCK) sm.acc[i / 5][i % 5] = 0ull;
-  const uint32_t per_group = a.n_chunks + a.n_tiles;
-  const uint32_t total = per_group * (uint32_t)a.G;
+  const int par = (level - 1) & 1;  // queues were produced by commit l-1 (or init)
+  if (tid == 0) {
+    uint32_t ph = 0, pl = 0;
+    for (int g = 0; g < a.G; ++g) {
+      const GroupCtrl<T> &c = a.ctrl[g];
+      sm.nitems[0][g] = ph;
+      sm.nitems[1][g] = pl;
+      if (!c.done) {
+        const int base = c.dir ? Q_BUL : Q_TDL;
+        const uint32_t qh = c.dir ? QBH : QH;
+        ph += (c.qlen[par][base + 1] + qh - 1) / qh;
+        pl += (c.qlen[par][base] + QL - 1) / QL;
+      }
+    }
+    sm.nitems[0][a.G] = ph;
+    sm.nitems[1][a.G] = pl;
+  }
+  __syncthreads();
+  const uint32_t n_hub = a.n_chunks * (uint32_t)a.G;
+  const uint32_t n_heavy = sm.nitems[0][a.G];
+  const uint32_t total = n_hub + n_heavy + sm.nitems[1][a.G];
+  uint32_t pending = 0;
+  if (tid == 0) pending = atomicAdd(a.work_ctr + level, 1u);
   for (;;) {
     __syncthreads();
-    if (tid == 0) sm.item = atomicAdd(a.work_ctr + level, 1u);
+    if (tid == 0) {
+      sm.item = pending;
+      if (pending < total) pending = atomicAdd(a.work_ctr + level, 1u);
+    }
     __syncthreads();
     const uint32_t item = sm.item;
     if (item >= total) break;
-    const int g = (int)(item % (uint32_t)a.G);
-    const uint32_t k = item / (uint32_t)a.G;
-    const GroupCtrl<T> *c = a.ctrl + g;
-    if (c->done) continue;
-    const uint32_t dir = c->dir;
-    if (k < a.n_chunks) {
-      const HubChunk hc = a.chunks[k];
-      if (dir == 0) hub_td<T>(a, sm, g, hc, level);
+    if (item < n_hub) {
+      const int g = (int)(item % (uint32_t)a.G);
+      const GroupCtrl<T> *c = a.ctrl + g;
+      if (c->done) continue;
+      const HubChunk hc = a.chunks[item / (uint32_t)a.G];
+      if (c->dir == 0) hub_td<T>(a, sm, g, hc, level);
       else hub_bu<T>(a, sm, s_red, g, hc, level, c->active);
-    } else if (dir == 0) {
-      tile_td<T>(a, sm, s_word, g, k - a.n_chunks, level);
-    } else {
-      tile_bu<T>(a, sm, s_word, g, k - a.n_chunks, level, c->active);
+      continue;
     }
+    const bool heavy = item < n_hub + n_heavy;
+    const int sel = heavy ? 0 : 1;
+    const uint32_t r = heavy ? item - n_hub : item - n_hub - n_heavy;
+    int g = 0;
+    while (g + 1 < a.G && sm.nitems[sel][g + 1] <= r) ++g;
+    const GroupCtrl<T> *c = a.ctrl + g;
+    const uint32_t k = r - sm.nitems[sel][g];
+    const int cls = (c->dir ? Q_BUL : Q_TDL) + (heavy ? 1 : 0);
+    const uint32_t qlen = c->qlen[par][cls];
+    const uint32_t per = c->dir ? (heavy ? QBH : QL) : (heavy ? QH : QL);
+    const uint32_t i0 = k * per, i1 = min(qlen, i0 + per);
+    if (c->dir == 0) item_td<T>(a, sm, tq, g, cls, i0, i1, level);
+    else item_bu<T>(a, sm, tq, g, cls, i0, i1, level, c->active);
   }
   __syncthreads();
   for (int i = tid; i < a.G; i += BLOCK) {
@@ -548,97 +705,139 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
   return s0 + (s1 << 16) + (s2 << 32) + (s3 << 48);
 }
 
-template <typename T>
 __device__ __forceinline__ bool decide_bu(const Policy &p, uint32_t next_level, uint32_t cur_dir,
-                                          unsigned long long n_f, unsigned long long m_f,
-                                          unsigned long long m_u) {
+                                          unsigned long long n_f, unsigned long long m_f) {
   if (p.mode == 1) return false;
   if (p.mode == 2) return next_level >= p.bu_from;
   if (p.mode == 3 && next_level - 1 < p.sched_len) return p.sched[next_level - 1] != 0;
-  // auto (reading #7): TD -> BU when the frontier's edges m_f exceed the
-  // unexplored edges m_u / alpha; BU -> TD when the frontier holds < nv_active / beta
-  // vertices.
-  if (cur_dir == 0) return (double)m_f * (double)p.alpha > (double)m_u && m_f > 0;
+  // auto (reading #7): TD -> BU when the edges of the next frontier, m_f,
+  // exceed ne / alpha (in joint BFS nearly every vertex keeps an unvisited active bit
+  // for several levels, so Beamer's unexplored-edge count m_u is ~ne); BU -> TD when the
+  // frontier holds fewer than nv_active / beta vertices.
+  if (cur_dir == 0) return m_f > 0 && (double)m_f * (double)p.alpha > (double)p.ne;
   return !((double)n_f * (double)p.beta < (double)p.nv_active);
 }
 
+// Commit of level l for one group (blockIdx.y): visited |= S_l, zero slot l+1, and
+// build both JFQs of level l+1 -- top-down: vertices with new bits; bottom-up: vertices
+// with an unvisited bit of an instance active before this level (a superset of the
+// active set after it: the expand masks with the final one, Lemma C3.5).
 template <typename T>
 __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level) {
-  constexpr int W = WordBits<T>::value;
-  constexpr int PIECES = W / 32;
-  __shared__ unsigned long long s_red[NWARP][4];
+  __shared__ unsigned long long s_red[NWARP][3];
   __shared__ T s_or[NWARP];
   __shared__ uint32_t s_last;
+  __shared__ uint32_t s_wcnt[NWARP][4];
+  __shared__ uint32_t s_qbase[4];
   const int g = blockIdx.y;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   GroupCtrl<T> *c = a.ctrl + g;
   if (*(volatile uint32_t *)&c->done) return;
   const T active = c->active;
   const T *N = next_buf(a, g, level);
-  T *F = frontier_buf(a, g, level);
+  T *Z = snap(a, g, level + 1);  // target of the next level's expand
   T *vis = a.visited + (size_t)g * a.gstride;
-  int8_t *out = a.out + (size_t)g * W * a.nv;
+  uint32_t *qlen = c->qlen[level & 1];
   const size_t nv = a.nv;
-  unsigned long long nf = 0, mf = 0, mu = 0, newp = 0;
+  unsigned long long nf = 0, mf = 0, newp = 0;
   T nacc = wzero_value<T>();
-  bool range = false;
   const size_t stride = (size_t)gridDim.x * BLOCK;
-  for (size_t base = (size_t)blockIdx.x * BLOCK; base < nv; base += stride) {
-    const size_t v = base + tid;
-    const bool in = v < nv;
-    T n = wzero_value<T>();
-    T vv = wzero_value<T>();
-    if (in) {
-      n = ld(N + v);
-      vv = ld(vis + v);
-      st(F + v, wzero_value<T>());
-    }
-    const bool nz = !wzero(n);
-    if (nz) st(vis + v, wor(vv, n));
-    const T tnew = in ? wandn(active, wor(vv, n)) : wzero_value<T>();
-    const bool un = !wzero(tnew);
-    const uint32_t d = (nz || un) ? __ldg(a.deg + v) : 0u;
-    if (nz) { nf++; mf += d; newp += wpopc(n); nacc = wor(nacc, n); }
-    if (un) mu += d;
-    if (level <= 127) {
-      // depth record: iterate the bits set anywhere in the warp so that lanes holding
-      // the same instance j store to consecutive bytes of row j together
+  // CVT vertices per thread per block iteration; the four queue classes are appended
+  // with one atomic per class per block iteration (block-wide ballot prefix).
+  constexpr int CVT = 4;
+  for (size_t base = (size_t)blockIdx.x * BLOCK * CVT; base < nv; base += stride * CVT) {
+    T n[CVT], vv[CVT];
+    uint32_t dg[CVT];
 #pragma unroll
-      for (int k = 0; k < PIECES; ++k) {
-        const uint32_t p = wpiece(n, k);
-        uint32_t any = __reduce_or_sync(FULL, p);
-        while (any) {
-          const int j = __ffs(any) - 1;
-          any &= any - 1;
-          if ((p >> j) & 1u) out[(size_t)(k * 32 + j) * nv + v] = (int8_t)level;
-        }
+    for (int k = 0; k < CVT; ++k) {
+      const size_t v = base + (size_t)k * BLOCK + tid;
+      n[k] = wzero_value<T>();
+      vv[k] = wzero_value<T>();
+      dg[k] = 0;
+      if (v < nv) {
+        // S_l is disjoint from visited: TD masked it with the committed words, BU with T.
+        n[k] = ld(N + v);
+        vv[k] = ld(vis + v);
+        dg[k] = __ldg(a.deg + v);
       }
-    } else if (nz) {
-      range = true;
     }
+    uint32_t bal[CVT][4];
+    uint32_t wc[4] = {0, 0, 0, 0};
+#pragma unroll
+    for (int k = 0; k < CVT; ++k) {
+      const size_t v = base + (size_t)k * BLOCK + tid;
+      const bool in = v < nv;
+      if (in) st(Z + v, wzero_value<T>());
+      const bool nz = !wzero(n[k]);
+      if (nz) st(vis + v, wor(vv[k], n[k]));
+      const T tp = in ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
+      const bool un = !wzero(tp);
+      const uint32_t d = dg[k];
+      if (nz) {
+        nf++;
+        mf += d;
+        newp += wpopc(n[k]);
+        nacc = wor(nacc, n[k]);
+      }
+      const bool qd = d > 0 && d <= (uint32_t)HUB_T;
+      const bool light = d <= (uint32_t)LIGHT_DEG;
+      bal[k][Q_TDL] = __ballot_sync(FULL, nz && qd && light);
+      bal[k][Q_TDH] = __ballot_sync(FULL, nz && qd && !light);
+      bal[k][Q_BUL] = __ballot_sync(FULL, un && qd && light);
+      bal[k][Q_BUH] = __ballot_sync(FULL, un && qd && !light);
+#pragma unroll
+      for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
+    }
+    if (lane == 0)
+      for (int cls = 0; cls < 4; ++cls) s_wcnt[warp][cls] = wc[cls];
+    __syncthreads();
+    if (tid < 4) {
+      uint32_t tot = 0;
+      for (int w = 0; w < NWARP; ++w) {
+        const uint32_t x = s_wcnt[w][tid];
+        s_wcnt[w][tid] = tot;  // exclusive warp offsets
+        tot += x;
+      }
+      s_qbase[tid] = tot ? atomicAdd(qlen + tid, tot) : 0u;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int cls = 0; cls < 4; ++cls) {
+      uint32_t off = s_qbase[cls] + s_wcnt[warp][cls];
+      uint32_t *q = queue_of(a, g, cls);
+#pragma unroll
+      for (int k = 0; k < CVT; ++k) {
+        const uint32_t b = bal[k][cls];
+        if ((b >> lane) & 1u) {
+          const uint32_t i = off + __popc(b & lanemask_lt());
+          const uint32_t v = (uint32_t)(base + (size_t)k * BLOCK + tid);
+          if (cls & 1) q[nv - 1 - i] = v; else q[i] = v;
+        }
+        off += __popc(b);
+      }
+    }
+    __syncthreads();  // s_wcnt / s_qbase reused next iteration
   }
-  if (range) atomicExch(a.range_err, 1u);
+  if (level >= 128 && !wzero(nacc)) atomicExch(a.range_err, 1u);  // depth > 127
   nf = warp_sum64(nf);
   mf = warp_sum64(mf);
-  mu = warp_sum64(mu);
   newp = warp_sum64(newp);
   nacc = warp_or(nacc);
   if (lane == 0) {
-    s_red[warp][0] = nf; s_red[warp][1] = mf; s_red[warp][2] = mu; s_red[warp][3] = newp;
+    s_red[warp][0] = nf; s_red[warp][1] = mf; s_red[warp][2] = newp;
     s_or[warp] = nacc;
   }
   __syncthreads();
   if (tid == 0) {
-    unsigned long long t0 = 0, t1 = 0, t2 = 0, t3 = 0;
+    unsigned long long t0 = 0, t1 = 0, t2 = 0;
     T o = wzero_value<T>();
     for (int k = 0; k < NWARP; ++k) {
-      t0 += s_red[k][0]; t1 += s_red[k][1]; t2 += s_red[k][2]; t3 += s_red[k][3];
+      t0 += s_red[k][0]; t1 += s_red[k][1]; t2 += s_red[k][2];
       o = wor(o, s_or[k]);
     }
     if (t0) atomicAdd(&c->n_f, t0);
     if (t1) atomicAdd(&c->m_f, t1);
-    if (t2) atomicAdd(&c->m_u, t2);
-    if (t3) atomicAdd(&c->newp, t3);
+    if (t2) atomicAdd(&c->newp, t2);
     if (!wzero(o)) red_or(&c->newacc, o);
     __threadfence();
     const uint32_t prev = atomicAdd(&c->arrive, 1u);
@@ -648,67 +847,157 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
   if (s_last && tid == 0) {
     __threadfence();
     const T act = ldv(&c->newacc);
-    const unsigned long long n_f = ldv(&c->n_f), m_f = ldv(&c->m_f), m_u = ldv(&c->m_u),
-                             np = ldv(&c->newp);
+    const unsigned long long n_f = ldv(&c->n_f), m_f = ldv(&c->m_f), np = ldv(&c->newp);
     const uint32_t cur = c->dir;
     LevelStat *ls = a.lstat + (size_t)g * MAXL + level;
     ls->dir = cur + 1;
     ls->newp = np;
     ls->nf = n_f;
-    const bool bu = decide_bu<T>(a.pol, (uint32_t)level + 1, cur, n_f, m_f, m_u);
+    const bool bu = decide_bu(a.pol, (uint32_t)level + 1, cur, n_f, m_f);
     c->active = act;
     c->newacc = wzero_value<T>();
-    c->n_f = c->m_f = c->m_u = c->newp = 0;
+    c->n_f = c->m_f = c->newp = 0;
     c->dir = bu ? 1u : 0u;
     c->arrive = 0;
     c->last_level = (uint32_t)level;
+    for (int k = 0; k < 4; ++k) c->qlen[(level + 1) & 1][k] = 0;  // target of commit l+1
     if (wzero(act)) {
       c->done = 1;
       __threadfence();
       atomicAdd(a.batch_done, 1u);
+    } else if (level + 1 < MAXL) {
+      // Eq. 1 counters of level l+1 known here: TD -- |JFQ| = vertices with new bits,
+      // sum_j |FQ_j| = new pairs; BU -- the isolated vertices (never in the queues; every
+      // active instance is unvisited there), the expand adds the queued ones and hubs.
+      LevelStat *nx = a.lstat + (size_t)g * MAXL + level + 1;
+      if (!bu) {
+        nx->jfq = n_f;
+        nx->fq = np;
+      } else {
+        nx->jfq = a.n_iso;
+        nx->fq = (unsigned long long)a.n_iso * (unsigned long long)wpopc(act);
+      }
     }
   }
 }
 
-// --------------------------------------------------------------------- finalize ----
-// m_s = sum over reached v of deg(v) (reading #11), from the final visited words.
+// ------------------------------------------------------------------------ depth ----
+// Depth rows from the level snapshots l in [l0, l1] (l1 capped at the group's last
+// committed level and at 127): depth[j][v] = the first l with bit j of S_l[v] set.
+// One CTA handles DT consecutive vertices x all W rows: each thread (= one vertex)
+// accumulates (l + 1) into the byte of every row whose bit first appears at level l
+// (4 rows per 32-bit register, SIMD-within-a-register: bytes never carry since each
+// receives at most one value <= 128), stores its bytes into a [W][DT] shared tile, and
+// the CTA writes the tile row by row with full 128-byte lines.  first != 0 writes every
+// byte (-1 where no bit was found); otherwise only the bytes found in [l0, l1] change.
+constexpr int DT = 128;
+
+__device__ __forceinline__ uint32_t spread4(uint32_t nib) {
+  // 4-bit nibble -> 0x01 in each byte whose bit is set
+  return (nib * 0x00204081u) & 0x01010101u;
+}
+
+// The same pass accumulates m_s (reading #11): every byte it finds adds deg(v) to row j's
+// sum (each (j, v) is found in exactly one flush), in shared memory per CTA, flushed to
+// m_out once per CTA.  CTAs loop over vertex tiles (grid = a few waves).
 template <typename T>
-__global__ void __launch_bounds__(BLOCK) msum_kernel(BatchArgs<T> a, unsigned long long *m_out) {
+__global__ void __launch_bounds__(DT) depth_kernel(BatchArgs<T> a, int l0, int l1, int first,
+                                                   unsigned long long *m_out) {
   constexpr int W = WordBits<T>::value;
-  constexpr int PIECES = W / 32;
+  constexpr int Q = W / 4;  // 32-bit registers of depth bytes per vertex
+  constexpr int ROWW = DT / 4 + 1;
+  constexpr int ROWB = ROWW * 4;
+  __shared__ __align__(16) uint32_t tile[W][ROWW];
+  __shared__ uint32_t s_deg[DT];
   __shared__ unsigned long long s_m[W];
   const int g = blockIdx.y;
-  const int tid = threadIdx.x, lane = tid & 31;
-  for (int j = tid; j < W; j += BLOCK) s_m[j] = 0;
-  __syncthreads();
-  const T *vis = a.visited + (size_t)g * a.gstride;
-  const size_t stride = (size_t)gridDim.x * BLOCK;
-  for (size_t base = (size_t)blockIdx.x * BLOCK; base < a.nv; base += stride) {
-    const size_t v = base + tid;
-    const bool in = v < a.nv;
-    const T vv = in ? ld(vis + v) : wzero_value<T>();
-    const uint32_t d = in ? __ldg(a.deg + v) : 0u;
+  const int rows = group_rows(a, g);
+  if (rows == 0) return;
+  const int t = threadIdx.x, lane = t & 31;
+  for (int j = t; j < W; j += DT) s_m[j] = 0;
+  const GroupCtrl<T> *c = a.ctrl + g;
+  const int last = min((int)c->last_level, min(l1, 127));
+  int8_t *out = a.out + (size_t)g * W * a.nv;
+  const size_t nvv = a.nv;
+  const size_t ntiles = (nvv + DT - 1) / DT;
+  unsigned char *tb = reinterpret_cast<unsigned char *>(&tile[0][0]);
+  const int8_t *tile_bytes = reinterpret_cast<const int8_t *>(tb);
+  for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x) {
+    const size_t v0 = tix * DT;
+    const size_t v = v0 + t;
+    const bool in = v < nvv;
+    uint32_t acc[Q];
 #pragma unroll
-    for (int k = 0; k < PIECES; ++k) {
-      const uint32_t p = wpiece(vv, k);
-      uint32_t any = __reduce_or_sync(FULL, p);
-      while (any) {
-        const int j = __ffs(any) - 1;
-        any &= any - 1;
-        const uint32_t x = ((p >> j) & 1u) ? d : 0u;
-        const unsigned long long s =
-            (unsigned long long)__reduce_add_sync(FULL, x & 0xffffu) +
-            ((unsigned long long)__reduce_add_sync(FULL, x >> 16) << 16);
-        if (lane == 0) atomicAdd(&s_m[k * 32 + j], s);
+    for (int q = 0; q < Q; ++q) acc[q] = 0;
+    if (in) {
+      T reached = wzero_value<T>();
+      for (int l = l0; l <= last; ++l) {
+        const T w = ld(snap(a, g, l) + v);
+        const T nb = wandn(w, reached);
+        if (wzero(nb)) continue;
+        reached = wor(reached, nb);
+        const uint32_t inc = (uint32_t)(l + 1);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+          const uint32_t nib = (wpiece(nb, q >> 3) >> ((q & 7) * 4)) & 0xFu;
+          acc[q] += spread4(nib) * inc;
+        }
+      }
+    }
+    __syncthreads();  // previous tile fully written out
+    s_deg[t] = in ? __ldg(a.deg + v) : 0u;
+#pragma unroll
+    for (int q = 0; q < Q; ++q) {
+      const uint32_t x = __vsub4(acc[q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
+#pragma unroll
+      for (int b = 0; b < 4; ++b) tb[(q * 4 + b) * ROWB + t] = (unsigned char)(x >> (8 * b));
+    }
+    __syncthreads();
+    const bool vec = first && ((nvv & 15) == 0) && (((uintptr_t)out & 15) == 0) && (v0 + DT <= nvv);
+    if (vec) {
+      // 8 threads x 16 bytes per 128-byte row segment; DT/8 = 16 rows per pass
+      const int sub = t & 7, r0 = t >> 3;
+      for (int j = r0; j < W; j += DT / 8) {  // all lanes iterate (shuffles below)
+        unsigned long long part = 0;
+        if (j < rows) {
+          const uint32_t *src = &tile[j][sub * 4];
+          const uint32_t x0 = src[0], x1 = src[1], x2 = src[2], x3 = src[3];
+          *reinterpret_cast<int4 *>(out + (size_t)j * nvv + v0 + sub * 16) =
+              make_int4((int)x0, (int)x1, (int)x2, (int)x3);
+          const uint32_t xs[4] = {x0, x1, x2, x3};
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+#pragma unroll
+            for (int b = 0; b < 4; ++b)
+              if (((xs[k] >> (8 * b)) & 0xffu) != 0xffu) part += s_deg[sub * 16 + k * 4 + b];
+        }
+        part += __shfl_xor_sync(FULL, part, 1);
+        part += __shfl_xor_sync(FULL, part, 2);
+        part += __shfl_xor_sync(FULL, part, 4);
+        if (sub == 0 && j < rows && part) atomicAdd(&s_m[j], part);
+      }
+    } else {
+      const size_t vv = v0 + t;
+      for (int j = 0; j < rows; ++j) {
+        const int8_t d = tile_bytes[j * ROWB + t];
+        unsigned long long part = 0;
+        if (vv < nvv && d != -1) {
+          out[(size_t)j * nvv + vv] = d;
+          part = s_deg[t];
+        } else if (vv < nvv && first) {
+          out[(size_t)j * nvv + vv] = d;
+        }
+        part = warp_sum64(part);
+        if (lane == 0 && part) atomicAdd(&s_m[j], part);
       }
     }
   }
   __syncthreads();
-  const int rows = group_rows(a, g);
-  for (int j = tid; j < rows; j += BLOCK)
+  for (int j = t; j < rows; j += DT)
     if (s_m[j]) atomicAdd(&m_out[(size_t)g * W + j], s_m[j]);
 }
 
+// --------------------------------------------------------------------- finalize ----
 __device__ __forceinline__ unsigned long long splitmix64(unsigned long long z) {
   z += 0x9E3779B97F4A7C15ull;
   z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;

@@ -79,12 +79,15 @@ class RunStats:
     expand_ms: float
     commit_ms: float
     init_ms: float
+    depth_ms: float
     expand_launches: int
     commit_launches: int
     init_launches: int
+    depth_launches: int
     expand_bytes: int
     commit_bytes: int
     init_bytes: int
+    depth_bytes: int
     per_source_m: np.ndarray | None = None
     per_source_digest: np.ndarray | None = None
     per_level: list = field(default_factory=list)
@@ -114,6 +117,11 @@ class Graph:
         self.nv, self.ne, self.max_degree = int(nv.value), int(ne.value), int(md.value)
 
     # ---- loading -------------------------------------------------------------------
+    def sort_rows(self, hub_first: bool = True) -> "Graph":
+        """ibfs_graph_sort_rows: neighbour lists by outdegree, descending (results unchanged)."""
+        check(_lib.load().ibfs_graph_sort_rows(self._h, _lib.ROWS_HUB_FIRST if hub_first else _lib.ROWS_KEEP))
+        return self
+
     @classmethod
     def from_csr(cls, offsets, adj, device: int = 0) -> "Graph":
         lib = _lib.load()
@@ -143,8 +151,9 @@ class Graph:
         return cls(h, device)
 
     @classmethod
-    def from_edgelist(cls, el, device: int = 0) -> "Graph":
-        return cls.from_edges(el.nv, el.u, el.v, device, getattr(el, "directed", False))
+    def from_edgelist(cls, el, device: int = 0, hub_first: bool = True) -> "Graph":
+        g = cls.from_edges(el.nv, el.u, el.v, device, getattr(el, "directed", False))
+        return g.sort_rows(True) if hub_first else g
 
     def close(self):
         if getattr(self, "_h", None):

@@ -234,13 +234,28 @@ def test_planner_matches_oracle_planner(W):
 
 def test_csr_build_matches_oracle_adjacency():
     el = ibfs_gen.rmat(12, 8, ibfs_gen.RMAT, seed=4)
-    g = P.Graph.from_edgelist(el)
+    g = P.Graph.from_edgelist(el, hub_first=False)
     off, adj = g.export_csr()
     ooff, oadj = oracle.OracleGraph.from_edges(el).adjacency()
     np.testing.assert_array_equal(off, ooff)
     np.testing.assert_array_equal(adj, oadj)  # tuple order kept within every row
     g2 = P.Graph.from_csr(off, adj)
     assert (g2.nv, g2.ne, g2.max_degree) == (g.nv, g.ne, g.max_degree)
+    # hub-first rows: same multiset per row, neighbour degree non-increasing, stable
+    g2.sort_rows(True)
+    off2, adj2 = g2.export_csr()
+    np.testing.assert_array_equal(off2, off)
+    deg = np.diff(off.astype(np.int64))
+    for v in range(0, el.nv, 7):
+        r0, r1 = int(off[v]), int(off[v + 1])
+        row, srow = adj[r0:r1], adj2[r0:r1]
+        assert sorted(row.tolist()) == sorted(srow.tolist())
+        exp = sorted(range(r1 - r0), key=lambda i: (-deg[row[i]], i))
+        np.testing.assert_array_equal(srow, row[exp])
+    s = np.arange(0, el.nv, 37, dtype=np.uint32)
+    d1, _ = g.run(s, 64)
+    d2, _ = g2.run(s, 64)
+    np.testing.assert_array_equal(d1.cpu().numpy(), d2.cpu().numpy())
 
 
 # --------------------------------------------------------------------- edge cases

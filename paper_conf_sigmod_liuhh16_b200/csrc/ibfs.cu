@@ -804,7 +804,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DT - 1) / DT,
                                                                          (uint64_t)g->num_sms * 16 / Gb + 1));
-      depth_kernel<T><<<dim3(bx, Gb), DT, 0, stream>>>(a, flushed + 1, l1, flushed < 0 ? 1 : 0, d_m);
+      depth_kernel<T><<<dim3(bx, Gb), DTHREADS, 0, stream>>>(a, flushed + 1, l1, flushed < 0 ? 1 : 0, d_m);
       if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
       launches++;
       st.depth_launches++;

@@ -897,24 +897,68 @@ __device__ __forceinline__ uint32_t spread4(uint32_t nib) {
   return (nib * 0x00204081u) & 0x01010101u;
 }
 
+// m16n8k32 u8 x u8 -> s32 tensor-core MMA (D += A * B), fragments per the PTX ISA.
+__device__ __forceinline__ void mma_u8_m16n8k32(int (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2,
+                                                uint32_t a3, uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k32.row.col.s32.u8.u8.s32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};\n"
+      : "+r"(d[0]), "+r"(d[1]), "+r"(d[2]), "+r"(d[3])
+      : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+
+// byte b of four consecutive degrees, packed little-endian
+__device__ __forceinline__ uint32_t byte_plane4(const uint32_t *d, int b) {
+  const int sh = 8 * b;
+  return ((d[0] >> sh) & 0xffu) | (((d[1] >> sh) & 0xffu) << 8) | (((d[2] >> sh) & 0xffu) << 16) |
+         (((d[3] >> sh) & 0xffu) << 24);
+}
+
+// add the MMA accumulators (rows 0..3 = byte planes; lanes with gq < 4) into s_m, reset
+template <int NT>
+__device__ __forceinline__ void flush_macc(int (&dacc)[NT][4], unsigned long long *s_m, int warp, int gq,
+                                           int tq4) {
+  if (gq < 4) {
+#pragma unroll
+    for (int nt = 0; nt < NT; ++nt) {
+      const int j0 = (warp * NT + nt) * 8 + tq4 * 2;
+      if (dacc[nt][0]) atomicAdd(&s_m[j0], (unsigned long long)(uint32_t)dacc[nt][0] << (8 * gq));
+      if (dacc[nt][1]) atomicAdd(&s_m[j0 + 1], (unsigned long long)(uint32_t)dacc[nt][1] << (8 * gq));
+    }
+  }
+#pragma unroll
+  for (int nt = 0; nt < NT; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
+}
+
 // The same pass accumulates m_s (reading #11): every byte it finds adds deg(v) to row j's
-// sum (each (j, v) is found in exactly one flush), in shared memory per CTA, flushed to
-// m_out once per CTA.  CTAs loop over vertex tiles (grid = a few waves).
+// sum (each (j, v) is found in exactly one flush) -- a [4 x DT] x [DT x W] u8 product per
+// tile on the tensor cores, flushed to m_out once per CTA.  CTAs loop over vertex tiles.
+constexpr int DTHREADS = DT;  // one thread per vertex of the tile
+
 template <typename T>
-__global__ void __launch_bounds__(DT) depth_kernel(BatchArgs<T> a, int l0, int l1, int first,
-                                                   unsigned long long *m_out) {
+__global__ void __launch_bounds__(DTHREADS) depth_kernel(BatchArgs<T> a, int l0, int l1, int first,
+                                                        unsigned long long *m_out) {
   constexpr int W = WordBits<T>::value;
   constexpr int Q = W / 4;  // 32-bit registers of depth bytes per vertex
   constexpr int ROWW = DT / 4 + 1;
   constexpr int ROWB = ROWW * 4;
+  constexpr int NWD = DTHREADS / 32;               // warps
+  constexpr int NTILES = W / 8;                    // 8-row n-tiles of the MMA
+  constexpr int NTW = NTILES >= NWD ? NTILES / NWD : 1;
+  constexpr int MMA_WARPS = NTILES / NTW;          // warps taking part in the MMA
   __shared__ __align__(16) uint32_t tile[W][ROWW];
   __shared__ uint32_t s_deg[DT];
   __shared__ unsigned long long s_m[W];
   const int g = blockIdx.y;
   const int rows = group_rows(a, g);
   if (rows == 0) return;
-  const int t = threadIdx.x, lane = t & 31;
-  for (int j = t; j < W; j += DT) s_m[j] = 0;
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  const int gq = lane >> 2, tq4 = lane & 3;  // mma fragment coordinates
+  int dacc[NTW][4];
+#pragma unroll
+  for (int nt = 0; nt < NTW; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
+  int tiles_acc = 0;
+  for (int j = t; j < W; j += DTHREADS) s_m[j] = 0;
   const GroupCtrl<T> *c = a.ctrl + g;
   const int last = min((int)c->last_level, min(l1, 127));
   int8_t *out = a.out + (size_t)g * W * a.nv;
@@ -932,8 +976,7 @@ __global__ void __launch_bounds__(DT) depth_kernel(BatchArgs<T> a, int l0, int l
     if (in) {
       T reached = wzero_value<T>();
       for (int l = l0; l <= last; ++l) {
-        const T w = ld(snap(a, g, l) + v);
-        const T nb = wandn(w, reached);
+        const T nb = wandn(ld(snap(a, g, l) + v), reached);
         if (wzero(nb)) continue;
         reached = wor(reached, nb);
         const uint32_t inc = (uint32_t)(l + 1);
@@ -953,47 +996,50 @@ __global__ void __launch_bounds__(DT) depth_kernel(BatchArgs<T> a, int l0, int l
       for (int b = 0; b < 4; ++b) tb[(q * 4 + b) * ROWB + t] = (unsigned char)(x >> (8 * b));
     }
     __syncthreads();
+    // m_s on the tensor cores: D[b][j] += sum_v deg_b(v) * reached(j, v), deg_b = byte b
+    // of deg(v) (A: 16 x 32 u8, rows 0..3 = byte planes), reached from the tile (B: 32 x 8
+    // u8, 0/1); m_s[j] = sum_b D[b][j] << 8b.
+    if (warp < MMA_WARPS) {
+#pragma unroll
+      for (int ks = 0; ks < DT / 32; ++ks) {
+        uint32_t a0 = 0, a2 = 0;
+        if (gq < 4) {
+          const int vb = ks * 32 + tq4 * 4;
+          a0 = byte_plane4(s_deg + vb, gq);
+          a2 = byte_plane4(s_deg + vb + 16, gq);
+        }
+#pragma unroll
+        for (int nt = 0; nt < NTW; ++nt) {
+          const int j = (warp * NTW + nt) * 8 + gq;
+          const uint32_t b0 = __vcmpne4(tile[j][ks * 8 + tq4], 0xffffffffu) & 0x01010101u;
+          const uint32_t b1 = __vcmpne4(tile[j][ks * 8 + 4 + tq4], 0xffffffffu) & 0x01010101u;
+          mma_u8_m16n8k32(dacc[nt], a0, 0u, a2, 0u, b0, b1);
+        }
+      }
+      if (++tiles_acc == 4096) {  // int32 headroom: <= 4 * 32 * 255 per tile and element
+        flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
+        tiles_acc = 0;
+      }
+    }
     const bool vec = first && ((nvv & 15) == 0) && (((uintptr_t)out & 15) == 0) && (v0 + DT <= nvv);
     if (vec) {
-      // 8 threads x 16 bytes per 128-byte row segment; DT/8 = 16 rows per pass
+      // 8 threads x 16 bytes per 128-byte row segment; DTHREADS/8 rows per pass
       const int sub = t & 7, r0 = t >> 3;
-      for (int j = r0; j < W; j += DT / 8) {  // all lanes iterate (shuffles below)
-        unsigned long long part = 0;
-        if (j < rows) {
-          const uint32_t *src = &tile[j][sub * 4];
-          const uint32_t x0 = src[0], x1 = src[1], x2 = src[2], x3 = src[3];
-          *reinterpret_cast<int4 *>(out + (size_t)j * nvv + v0 + sub * 16) =
-              make_int4((int)x0, (int)x1, (int)x2, (int)x3);
-          const uint32_t xs[4] = {x0, x1, x2, x3};
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-#pragma unroll
-            for (int b = 0; b < 4; ++b)
-              if (((xs[k] >> (8 * b)) & 0xffu) != 0xffu) part += s_deg[sub * 16 + k * 4 + b];
-        }
-        part += __shfl_xor_sync(FULL, part, 1);
-        part += __shfl_xor_sync(FULL, part, 2);
-        part += __shfl_xor_sync(FULL, part, 4);
-        if (sub == 0 && j < rows && part) atomicAdd(&s_m[j], part);
+      for (int j = r0; j < rows; j += DTHREADS / 8) {
+        const uint32_t *src = &tile[j][sub * 4];
+        *reinterpret_cast<int4 *>(out + (size_t)j * nvv + v0 + sub * 16) =
+            make_int4((int)src[0], (int)src[1], (int)src[2], (int)src[3]);
       }
-    } else {
-      const size_t vv = v0 + t;
+    } else if (v < nvv) {
       for (int j = 0; j < rows; ++j) {
         const int8_t d = tile_bytes[j * ROWB + t];
-        unsigned long long part = 0;
-        if (vv < nvv && d != -1) {
-          out[(size_t)j * nvv + vv] = d;
-          part = s_deg[t];
-        } else if (vv < nvv && first) {
-          out[(size_t)j * nvv + vv] = d;
-        }
-        part = warp_sum64(part);
-        if (lane == 0 && part) atomicAdd(&s_m[j], part);
+        if (first || d != -1) out[(size_t)j * nvv + v] = d;
       }
     }
   }
+  if (warp < MMA_WARPS) flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
   __syncthreads();
-  for (int j = t; j < rows; j += DT)
+  for (int j = t; j < rows; j += DTHREADS)
     if (s_m[j]) atomicAdd(&m_out[(size_t)g * W + j], s_m[j]);
 }
 

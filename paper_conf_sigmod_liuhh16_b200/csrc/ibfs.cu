@@ -158,18 +158,28 @@ bool is_device_ptr(const void *p) {
 }  // namespace
 
 // -------------------------------------------------------------------------- graph ----
+// The device graph lives in a compacted vertex space: the vertices of degree > 0, in the
+// caller's id order (compacted id = rank among them).  Isolated vertices never hold a
+// status word, never enter a queue and are never read by a level kernel; their depth
+// rows are written directly (-1, or 0 at an isolated source).  Because the ranks keep
+// the caller's order, adjacency rows keep their order and every "lower id" tie-break is
+// unchanged.
 struct ibfs_graph {
   int device = 0;
-  uint32_t nv = 0;
+  uint32_t nv = 0;          // caller's vertices
+  uint32_t nva = 0;         // vertices of degree > 0 (the compacted space)
   uint64_t ne = 0;
   uint32_t max_deg = 0;
-  uint64_t nv_active = 0;
-  unsigned long long *d_off = nullptr;
-  uint32_t *d_adj = nullptr;
-  uint32_t *d_deg = nullptr;
+  uint64_t nv_active = 0;   // = nva
+  unsigned long long *d_off = nullptr;  // [nva + 1]
+  uint32_t *d_adj = nullptr;            // [ne] compacted ids
+  uint32_t *d_deg = nullptr;            // [nva]
+  uint32_t *d_tbase = nullptr;          // [nv/128 + 1]: vertices of degree > 0 before tile t
+  uint32_t *d_nzbits = nullptr;         // [nv/32]: bit v%32 of word v/32 = (deg(v) > 0)
   HubChunk *d_chunks = nullptr;
   uint32_t n_chunks = 0;
-  std::vector<uint64_t> h_off;  // host copy (tiling, planner)
+  std::vector<uint64_t> h_off;      // host copy of d_off (tiling, planner)
+  std::vector<uint32_t> h_tbase, h_nzbits;
   int num_sms = 148;
   int expand_blocks_per_sm = 1;
 };
@@ -184,6 +194,8 @@ void graph_release(ibfs_graph *g) {
   cudaFree(g->d_adj);
   cudaFree(g->d_deg);
   cudaFree(g->d_chunks);
+  cudaFree(g->d_tbase);
+  cudaFree(g->d_nzbits);
   if (prev >= 0) cudaSetDevice(prev);
   cudaGetLastError();
   delete g;
@@ -217,11 +229,103 @@ __global__ void max_id_kernel(const uint32_t *adj, unsigned long long ne, uint32
   if ((threadIdx.x & 31) == 0) atomicMax(mx, m);
 }
 
+// ---- compaction ----
+__global__ void nzbits_kernel(const unsigned long long *off, uint32_t nv, uint32_t *nzbits) {
+  const size_t nvr = ((size_t)nv + 31) & ~(size_t)31;
+  for (size_t v = (size_t)blockIdx.x * blockDim.x + threadIdx.x; v < nvr; v += (size_t)gridDim.x * blockDim.x) {
+    const bool nz = v < nv && off[v + 1] > off[v];
+    const uint32_t b = __ballot_sync(FULL, nz);
+    if ((threadIdx.x & 31) == 0) nzbits[v >> 5] = b;
+  }
+}
+
+__global__ void tilecount_kernel(const uint32_t *nzbits, uint32_t nwords, uint32_t ntiles, uint32_t *cnt) {
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x) {
+    uint32_t c = 0;
+    for (uint32_t k = 4 * t; k < min(4 * t + 4, nwords); ++k) c += __popc(nzbits[k]);
+    cnt[t] = c;
+  }
+}
+
+__device__ __forceinline__ uint32_t dev_compact_id(const uint32_t *tbase, const uint32_t *nzbits, uint32_t v) {
+  const uint32_t w = v >> 5;
+  uint32_t c = tbase[v >> 7];
+  for (uint32_t k = w & ~3u; k < w; ++k) c += __popc(nzbits[k]);
+  return c + __popc(nzbits[w] & ((1u << (v & 31)) - 1u));
+}
+
+__global__ void compact_rows_kernel(const unsigned long long *off, uint32_t nv, const uint32_t *tbase,
+                                    const uint32_t *nzbits, unsigned long long *off_c) {
+  for (size_t v = (size_t)blockIdx.x * blockDim.x + threadIdx.x; v < nv; v += (size_t)gridDim.x * blockDim.x) {
+    if ((nzbits[v >> 5] >> (v & 31)) & 1u) off_c[dev_compact_id(tbase, nzbits, (uint32_t)v)] = off[v];
+  }
+}
+
+__global__ void remap_adj_kernel(uint32_t *adj, unsigned long long ne, const uint32_t *tbase, const uint32_t *nzbits) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < ne;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    adj[i] = dev_compact_id(tbase, nzbits, adj[i]);
+}
+
+// d_off_orig [nv + 1] (caller ids, consumed and freed) and g->d_adj (caller ids, remapped in
+// place) -> compacted g->d_off, g->d_adj, g->d_tbase, g->d_nzbits, host copies.
+void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig) {
+  const uint32_t nv = g->nv;
+  const uint32_t nwords = (nv + 31) / 32, ntiles = (nv + 127) / 128;
+  CK(cudaMalloc(&g->d_nzbits, std::max<size_t>(nwords, 1) * 4));
+  CK(cudaMalloc(&g->d_tbase, ((size_t)ntiles + 1) * 4));
+  uint32_t *cnt = nullptr;
+  void *tmp = nullptr;
+  try {
+    CK(cudaMalloc(&cnt, ((size_t)ntiles + 1) * 4));
+    CK(cudaMemset(cnt, 0, ((size_t)ntiles + 1) * 4));
+    nzbits_kernel<<<2048, 256>>>(d_off_orig, nv, g->d_nzbits);
+    tilecount_kernel<<<(ntiles + 255) / 256, 256>>>(g->d_nzbits, nwords, ntiles, cnt);
+    CK(cudaGetLastError());
+    size_t tb = 0;
+    CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, g->d_tbase, (int64_t)ntiles + 1));
+    CK(cudaMalloc(&tmp, std::max<size_t>(tb, 256)));
+    CK(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, g->d_tbase, (int64_t)ntiles + 1));
+    g->h_tbase.resize((size_t)ntiles + 1);
+    g->h_nzbits.resize(nwords);
+    CK(cudaMemcpy(g->h_tbase.data(), g->d_tbase, ((size_t)ntiles + 1) * 4, cudaMemcpyDeviceToHost));
+    if (nwords) CK(cudaMemcpy(g->h_nzbits.data(), g->d_nzbits, (size_t)nwords * 4, cudaMemcpyDeviceToHost));
+    g->nva = g->h_tbase[ntiles];
+    CK(cudaMalloc(&g->d_off, ((size_t)g->nva + 1) * sizeof(unsigned long long)));
+    const unsigned long long ne = g->ne;
+    CK(cudaMemcpy(g->d_off + g->nva, &ne, sizeof(ne), cudaMemcpyHostToDevice));
+    compact_rows_kernel<<<2048, 256>>>(d_off_orig, nv, g->d_tbase, g->d_nzbits, g->d_off);
+    if (g->ne) remap_adj_kernel<<<4096, 256>>>(g->d_adj, g->ne, g->d_tbase, g->d_nzbits);
+    CK(cudaGetLastError());
+    CK(cudaDeviceSynchronize());
+  } catch (...) {
+    cudaFree(cnt);
+    cudaFree(tmp);
+    cudaFree(d_off_orig);
+    throw;
+  }
+  cudaFree(cnt);
+  cudaFree(tmp);
+  cudaFree(d_off_orig);
+  g->h_off.resize((size_t)g->nva + 1);
+  CK(cudaMemcpy(g->h_off.data(), g->d_off, ((size_t)g->nva + 1) * 8, cudaMemcpyDeviceToHost));
+}
+
+// Host twin of compact_id for a caller id; NO_VERTEX if the vertex is isolated.
+uint32_t host_compact_id(const ibfs_graph *g, uint32_t v) {
+  const uint32_t w = v >> 5;
+  const uint32_t bits = g->h_nzbits[w];
+  if (!((bits >> (v & 31)) & 1u)) return NO_VERTEX;
+  uint32_t c = g->h_tbase[v >> 7];
+  for (uint32_t k = w & ~3u; k < w; ++k) c += (uint32_t)__builtin_popcount(g->h_nzbits[k]);
+  return c + (uint32_t)__builtin_popcount(bits & ((1u << (v & 31)) - 1u));
+}
+
 // Static hub decomposition: the rows of vertices with degree > HUB_T are
 // cut into chunks of CHUNK edges, each a work item a whole CTA sweeps.
 void build_decomposition(ibfs_graph *g) {
   std::vector<HubChunk> chunks;
-  for (uint32_t v = 0; v < g->nv; ++v) {
+  for (uint32_t v = 0; v < g->nva; ++v) {
     const uint64_t d = g->h_off[v + 1] - g->h_off[v];
     if (d <= (uint64_t)HUB_T) continue;
     uint32_t first = 1;
@@ -241,18 +345,18 @@ void build_decomposition(ibfs_graph *g) {
     CK(cudaMemcpy(g->d_chunks, chunks.data(), chunks.size() * sizeof(HubChunk), cudaMemcpyHostToDevice));
 }
 
-// Degrees, max degree, hub chunks; offsets must be in g->d_off and g->h_off.
+// Degrees, max degree, hub chunks; compacted offsets must be in g->d_off and g->h_off.
 void finish_graph(ibfs_graph *g) {
-  CK(cudaMalloc(&g->d_deg, std::max<size_t>(g->nv, 1) * sizeof(uint32_t)));
+  CK(cudaMalloc(&g->d_deg, std::max<size_t>(g->nva, 1) * sizeof(uint32_t)));
   unsigned long long *d_stats = nullptr;
   CK(cudaMalloc(&d_stats, 2 * sizeof(unsigned long long)));
   CK(cudaMemset(d_stats, 0, 2 * sizeof(unsigned long long)));
-  degree_kernel<<<1024, 256>>>(g->d_off, g->nv, g->d_deg, d_stats);
+  degree_kernel<<<1024, 256>>>(g->d_off, g->nva, g->d_deg, d_stats);
   CK(cudaGetLastError());
   unsigned long long h[2];
   CK(cudaMemcpy(h, d_stats, sizeof(h), cudaMemcpyDeviceToHost));
   cudaFree(d_stats);
-  for (uint32_t v = 0; v < g->nv; ++v)
+  for (uint32_t v = 0; v < g->nva; ++v)
     if (g->h_off[v + 1] - g->h_off[v] > 0xffffffffull)
       fail(IBFS_E_UNSUPPORTED, "vertex degree >= 2^32");
   g->max_deg = (uint32_t)h[0];
@@ -266,6 +370,12 @@ void finish_graph(ibfs_graph *g) {
                           (int)sizeof(TileQueue<unsigned long long>)));
   CK(cudaFuncSetAttribute(expand_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)sizeof(TileQueue<u128>)));
+  CK(cudaFuncSetAttribute(depth_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)depth_smem_bytes<uint32_t>()));
+  CK(cudaFuncSetAttribute(depth_kernel<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)depth_smem_bytes<unsigned long long>()));
+  CK(cudaFuncSetAttribute(depth_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)depth_smem_bytes<u128>()));
   int occ = 1;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, expand_kernel<u128>, BLOCK, sizeof(TileQueue<u128>)));
   g->expand_blocks_per_sm = std::max(1, occ);
@@ -320,8 +430,13 @@ extern "C" int ibfs_load_csr(int device, uint32_t nv, uint64_t ne, const uint64_
       if (g->h_off[0] != 0 || g->h_off[nv] != ne) fail(IBFS_E_INVALID, "offsets[0] != 0 or offsets[nv] != ne");
       for (uint32_t v = 0; v < nv; ++v)
         if (g->h_off[v + 1] < g->h_off[v]) fail(IBFS_E_INVALID, "offsets not non-decreasing");
-      CK(cudaMalloc(&g->d_off, ((size_t)nv + 1) * sizeof(unsigned long long)));
-      CK(cudaMemcpy(g->d_off, g->h_off.data(), ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
+      unsigned long long *d_off_orig = nullptr;
+      CK(cudaMalloc(&d_off_orig, ((size_t)nv + 1) * sizeof(unsigned long long)));
+      {
+        cudaError_t e = cudaMemcpy(d_off_orig, g->h_off.data(), ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) { cudaFree(d_off_orig); CK(e); }
+      }
+      g->d_off = d_off_orig;  // released by graph_release if a later step fails
       CK(cudaMalloc(&g->d_adj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
       if (ne) CK(cudaMemcpy(g->d_adj, adj, ne * sizeof(uint32_t), cudaMemcpyDefault));
       if (ne) {
@@ -335,6 +450,8 @@ extern "C" int ibfs_load_csr(int device, uint32_t nv, uint64_t ne, const uint64_
         cudaFree(d_mx);
         if (mx >= nv) fail(IBFS_E_INVALID, "adjacency id >= nv");
       }
+      g->d_off = nullptr;
+      compact_graph(g, d_off_orig);
       finish_graph(g);
     } catch (...) {
       graph_release(g);
@@ -388,12 +505,12 @@ extern "C" int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const
       cudaFree(d_u);
       cudaFree(d_v);
       tmp[0] = tmp[1] = nullptr;
-      CK(cudaMalloc(&g->d_off, ((size_t)nv + 1) * sizeof(unsigned long long)));
+      unsigned long long *d_off_orig = (unsigned long long *)dalloc(((size_t)nv + 1) * sizeof(unsigned long long));
       {  // offsets = exclusive scan of degrees (deg[nv] = 0 gives offsets[nv] = ne)
         size_t tb = 0;
-        CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, g->d_off, (int64_t)nv + 1));
+        CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, d_off_orig, (int64_t)nv + 1));
         void *t = dalloc(tb);
-        CK(cub::DeviceScan::ExclusiveSum(t, tb, deg, g->d_off, (int64_t)nv + 1));
+        CK(cub::DeviceScan::ExclusiveSum(t, tb, deg, d_off_orig, (int64_t)nv + 1));
       }
       CK(cudaMalloc(&g->d_adj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
       if (ne) {  // stable radix sort of (src, dst) by src keeps tuple order within rows
@@ -405,10 +522,10 @@ extern "C" int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const
         CK(cub::DeviceRadixSort::SortPairs(t, tb, keys_a, keys_b, vals_a, g->d_adj, (int64_t)ne, 0, bits));
       }
       CK(cudaDeviceSynchronize());
-      g->h_off.resize((size_t)nv + 1);
-      CK(cudaMemcpy(g->h_off.data(), g->d_off, ((size_t)nv + 1) * 8, cudaMemcpyDeviceToHost));
-      for (void *p : tmp) cudaFree(p);
+      for (void *&p : tmp)
+        if (p != d_off_orig) { cudaFree(p); p = nullptr; }
       tmp.clear();
+      compact_graph(g, d_off_orig);  // frees d_off_orig
       finish_graph(g);
     } catch (...) {
       for (void *p : tmp) cudaFree(p);
@@ -444,9 +561,9 @@ extern "C" int ibfs_graph_sort_rows(ibfs_graph *g, int order) {
     unsigned long long maxb = 0;
     std::vector<std::pair<uint32_t, uint32_t>> batches;
     uint32_t r0 = 0;
-    while (r0 < g->nv) {
+    while (r0 < g->nva) {
       uint32_t r1 = r0;
-      while (r1 < g->nv && g->h_off[r1 + 1] - g->h_off[r0] <= cap) ++r1;
+      while (r1 < g->nva && g->h_off[r1 + 1] - g->h_off[r0] <= cap) ++r1;
       if (r1 == r0) ++r1;  // a single row longer than cap (degree > 2^30): not expected
       batches.push_back({r0, r1});
       maxb = std::max<unsigned long long>(maxb, g->h_off[r1] - g->h_off[r0]);
@@ -512,8 +629,20 @@ extern "C" int ibfs_graph_export_csr(const ibfs_graph *g, uint64_t *offsets, uin
   return guarded([&] {
     if (!g || !offsets || (g->ne && !adj)) fail(IBFS_E_INVALID, "NULL argument");
     DeviceScope ds(g->device);
-    CK(cudaMemcpy(offsets, g->d_off, ((size_t)g->nv + 1) * 8, cudaMemcpyDeviceToHost));
-    if (g->ne) CK(cudaMemcpy(adj, g->d_adj, g->ne * 4, cudaMemcpyDeviceToHost));
+    // back to caller ids: offsets[v] = compacted offset of the first vertex of degree > 0
+    // at or after v (isolated rows are empty); adjacency ids through the inverse rank map
+    std::vector<uint32_t> orig;
+    orig.reserve(g->nva);
+    for (uint32_t v = 0; v < g->nv; ++v)
+      if ((g->h_nzbits[v >> 5] >> (v & 31)) & 1u) orig.push_back(v);
+    for (uint32_t v = 0, r = 0; v <= g->nv; ++v) {
+      offsets[v] = g->h_off[r];
+      if (v < g->nv && ((g->h_nzbits[v >> 5] >> (v & 31)) & 1u)) ++r;
+    }
+    if (g->ne) {
+      CK(cudaMemcpy(adj, g->d_adj, g->ne * 4, cudaMemcpyDeviceToHost));
+      for (uint64_t i = 0; i < g->ne; ++i) adj[i] = orig[adj[i]];
+    }
   });
 }
 
@@ -541,6 +670,10 @@ __global__ void hub_kernel(const unsigned long long *off, const uint32_t *adj, c
   const uint32_t warps = (gridDim.x * blockDim.x) >> 5;
   for (uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; r < n; r += warps) {
     const uint32_t s = src[r];
+    if (s == NO_VERTEX) {  // isolated source: no hub, degree 0
+      if (lane == 0) { hub[r] = 0xffffffffu; sdeg[r] = 0; }
+      continue;
+    }
     const unsigned long long e0 = off[s], e1 = off[s + 1];
     unsigned long long best = 0;
     bool have = false;
@@ -596,6 +729,7 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
     CK(cudaMemcpy(hsrc.data(), sources, (size_t)n * 4, cudaMemcpyDefault));
     for (uint32_t r = 0; r < n; ++r)
       if (hsrc[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
+    for (uint32_t r = 0; r < n; ++r) hsrc[r] = host_compact_id(g, hsrc[r]);  // planner works on compacted ids
     std::vector<uint32_t> hub(n, 0xffffffffu), sdeg(n, 0);
     if (pp.mode == 0) {
       uint32_t *d_src = nullptr, *d_hub = nullptr, *d_sdeg = nullptr;
@@ -673,12 +807,12 @@ struct EventTimer {
 };
 
 template <typename T>
-void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t *out_depths,
-               const ibfs_run_opts &o, ibfs_stats *stats) {
+void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *csources, uint32_t n,
+               int8_t *out_depths, const ibfs_run_opts &o, ibfs_stats *stats) {
   constexpr int W = WordBits<T>::value;
   constexpr size_t B = sizeof(T);
   cudaStream_t stream = (cudaStream_t)o.cuda_stream;
-  const uint32_t nv = g->nv;
+  const uint32_t nv = g->nv, nva = g->nva;
   const uint32_t n_groups = (n + W - 1) / W;
   const bool out_dev = is_device_ptr(out_depths);
   const bool out_host = out_depths && !out_dev;
@@ -686,18 +820,18 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   // groups per launch batch
   uint32_t G = o.groups_in_flight;
   if (G == 0) {
-    uint64_t want = (4ull << 20) / std::max<uint32_t>(nv, 1) + 1;
+    uint64_t want = (4ull << 20) / std::max<uint32_t>(nva, 1) + 1;
     G = (uint32_t)std::min<uint64_t>(want, MAX_G);
   }
   G = std::max<uint32_t>(1, std::min<uint32_t>({G, (uint32_t)MAX_G, n_groups}));
-  const size_t gstride = ((size_t)nv + 15) & ~(size_t)15;
+  const size_t gstride = ((size_t)nva + 16) & ~(size_t)15;
   const size_t rows_bytes_per_group = (size_t)W * nv;
   size_t free_b = 0, total_b = 0;
   CK(cudaMemGetInfo(&free_b, &total_b));
   // memory: visited + R snapshot slots per group (+ device rows if the caller's buffer
   // is not on the device); R >= 4, up to one slot per level when memory allows
   auto need = [&](uint32_t gg, uint32_t r) {
-    return gg * ((1 + r) * gstride * B + 8 * (size_t)nv + (out_dev ? 0 : rows_bytes_per_group)) + (size_t)n * 24;
+    return gg * ((1 + r) * gstride * B + 8 * (size_t)nva + (out_dev ? 0 : rows_bytes_per_group)) + (size_t)n * 28;
   };
   // The budget depends on the device size only (not on the momentary free memory), so
   // repeated calls request identical scratch and the stream-ordered pool reuses it.
@@ -710,10 +844,12 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   Scratch sc(g->device, stream);
   uint32_t *d_src = sc.get<uint32_t>(n);
   CK(cudaMemcpyAsync(d_src, sources, (size_t)n * 4, cudaMemcpyDefault, stream));
+  uint32_t *d_csrc = sc.get<uint32_t>(n);
+  CK(cudaMemcpyAsync(d_csrc, csources, (size_t)n * 4, cudaMemcpyDefault, stream));
   T *visited = sc.get<T>(G * gstride);
   T *ring = sc.get<T>((size_t)R * G * gstride);
-  uint32_t *tdq = sc.get<uint32_t>((size_t)G * nv);
-  uint32_t *buq = sc.get<uint32_t>((size_t)G * nv);
+  uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
+  uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
   LevelStat *lstat = sc.get<LevelStat>((size_t)G * MAXL);
   uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
@@ -733,7 +869,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   a.off = g->d_off;
   a.adj = g->d_adj;
   a.deg = g->d_deg;
+  a.tbase = g->d_tbase;
+  a.nzbits = g->d_nzbits;
   a.nv = nv;
+  a.nva = nva;
   a.gstride = gstride;
   a.visited = visited;
   a.ring = ring;
@@ -749,7 +888,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
   a.n_chunks = g->n_chunks;
   a.tdq = tdq;
   a.buq = buq;
-  a.n_iso = (uint32_t)(nv - g->nv_active);
+  a.n_iso = nv - nva;
   a.pol.mode = o.direction;
   a.pol.bu_from = o.bu_from;
   a.pol.alpha = o.alpha;
@@ -776,6 +915,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
     a.G = (int)Gb;
     a.group0 = gb0;
     a.src = d_src + (size_t)gb0 * W;
+    a.csrc = d_csrc + (size_t)gb0 * W;
     a.out = out_dev ? out_depths + (size_t)gb0 * rows_bytes_per_group : staging;
     const uint32_t rows_in_batch = std::min<uint32_t>(Gb * W, n - gb0 * W);
     CK(cudaMemsetAsync(flags, 0, 4, stream));
@@ -785,30 +925,30 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
     {
       cudaEvent_t i0 = nullptr, i1 = nullptr;
       if (o.timing) { i0 = timer.next(); i1 = timer.next(); CK(cudaEventRecord(i0, stream)); }
-      uint32_t bx = (uint32_t)std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, std::max<uint32_t>(1, 2048 / Gb));
+      uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nva + BLOCK - 1) / BLOCK, std::max<uint32_t>(1, 2048 / Gb)));
       init_ctrl_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
       init_state_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a, first_dir);
       init_sources_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
       CK(cudaGetLastError());
       launches += 3;
       st.init_launches += 3;
-      st.init_bytes += (uint64_t)Gb * (3 * nv * B);
+      st.init_bytes += (uint64_t)Gb * (3 * (uint64_t)nva * B);
       if (o.timing) { CK(cudaEventRecord(i1, stream)); kinit.push_back({i0, i1}); }
     }
     const uint32_t commit_bx = (uint32_t)std::max<uint64_t>(
-        1, std::min<uint64_t>(((uint64_t)nv + BLOCK - 1) / BLOCK, (uint64_t)g->num_sms * 8 / Gb));
+        1, std::min<uint64_t>(((uint64_t)nva + BLOCK * 4 - 1) / (BLOCK * 4), (uint64_t)g->num_sms * 8 / Gb));
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
     auto flush = [&](int l1) {
       cudaEvent_t d0 = nullptr, d1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
-      const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DT - 1) / DT,
-                                                                         (uint64_t)g->num_sms * 16 / Gb + 1));
-      depth_kernel<T><<<dim3(bx, Gb), DTHREADS, 0, stream>>>(a, flushed + 1, l1, flushed < 0 ? 1 : 0, d_m);
+      const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
+                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * 3 / Gb)));
+      depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, flushed < 0 ? 1 : 0, d_m);
       if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
       launches++;
       st.depth_launches++;
-      st.depth_bytes += (uint64_t)Gb * nv * (B * (uint64_t)(l1 - flushed)) + (uint64_t)rows_in_batch * nv;
+      st.depth_bytes += (uint64_t)Gb * nva * (B * (uint64_t)(l1 - flushed)) + (uint64_t)rows_in_batch * nv;
       flushed = l1;
     };
     int level = 1;
@@ -905,7 +1045,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n, int8_t 
         // inspection the adjacency entry and the neighbour's word; per write one word.
         // commit: S_l, visited and the zeroed slot streamed, visited written where new.
         uint64_t eb = (16 + B) * L.proc + (4 + B) * L.insp + B * L.writes;
-        uint64_t cb = (uint64_t)nv * (3 * B + 4) + B * L.nf;
+        uint64_t cb = (uint64_t)nva * (3 * B + 4) + B * L.nf;
         st.expand_bytes += eb;
         st.commit_bytes += cb;
       }
@@ -971,13 +1111,14 @@ extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_
     }
     DeviceScope ds(g->device);
     // sources: validate on the host
-    std::vector<uint32_t> hs(n);
+    std::vector<uint32_t> hs(n), hcs(n);
     CK(cudaMemcpy(hs.data(), sources, (size_t)n * 4, cudaMemcpyDefault));
     for (uint32_t r = 0; r < n; ++r)
       if (hs[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
-    if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), n, out_depths, o, stats);
-    else if (group_bits == 64) run_typed<unsigned long long>(g, hs.data(), n, out_depths, o, stats);
-    else run_typed<u128>(g, hs.data(), n, out_depths, o, stats);
+    for (uint32_t r = 0; r < n; ++r) hcs[r] = host_compact_id(g, hs[r]);
+    if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
+    else if (group_bits == 64) run_typed<unsigned long long>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
+    else run_typed<u128>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
   });
 }
 

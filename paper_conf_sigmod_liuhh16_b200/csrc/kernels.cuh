@@ -75,7 +75,6 @@ struct GroupCtrl {
   uint32_t done;
   uint32_t arrive;
   uint32_t last_level;
-  uint32_t iso_jfq1, iso_fq1;  // isolated-vertex part of a bottom-up level 1 (stats)
 };
 
 struct Policy {
@@ -90,16 +89,19 @@ struct Policy {
 
 template <typename T>
 struct BatchArgs {
-  const unsigned long long *off;
+  const unsigned long long *off;  // compacted CSR (vertices of degree > 0 only)
   const uint32_t *adj;
   const uint32_t *deg;
-  uint32_t nv;
+  const uint32_t *tbase;   // [nv/128 + 1] non-isolated vertices before each 128-vertex tile
+  const uint32_t *nzbits;  // [nv/32] bit v%32 of word v/32: vertex v has degree > 0
+  uint32_t nv;     // vertices of the caller's graph (depth row length)
+  uint32_t nva;    // non-isolated vertices (status word arrays, queues)
   size_t gstride;  // words per per-group array
   T *visited;
   T *ring;       // [R][gcap][gstride] level snapshots
   int R;         // ring slots
   int gcap;      // groups allocated per slot
-  uint32_t *tdq, *buq;  // [gcap][nv] queues
+  uint32_t *tdq, *buq;  // [gcap][nva] queues
   GroupCtrl<T> *ctrl;
   LevelStat *lstat;     // [G][MAXL]
   uint32_t *work_ctr;   // [MAXL]
@@ -108,13 +110,16 @@ struct BatchArgs {
   int G;
   uint32_t n_total;     // sources in the whole run
   uint32_t group0;      // global index of this batch's first group
-  const uint32_t *src;  // this batch's sources, group-major, row g*W + j
+  const uint32_t *src;  // this batch's sources (caller ids), group-major, row g*W + j
+  const uint32_t *csrc; // the same in compacted ids (NO_VERTEX if the source is isolated)
   int8_t *out;          // row g*W + j of this batch at out + (g*W + j) * nv
   const HubChunk *chunks;
   uint32_t n_chunks;
-  uint32_t n_iso;       // vertices of degree 0
+  uint32_t n_iso;       // vertices of degree 0 (nv - nva)
   Policy pol;
 };
+
+constexpr uint32_t NO_VERTEX = 0xffffffffu;
 
 template <typename T>
 __device__ __forceinline__ int group_rows(const BatchArgs<T> &a, int g) {
@@ -137,12 +142,12 @@ __device__ __forceinline__ T *next_buf(const BatchArgs<T> &a, int g, int level) 
 }
 template <typename T>
 __device__ __forceinline__ uint32_t *queue_of(const BatchArgs<T> &a, int g, int cls) {
-  return (cls < Q_BUL ? a.tdq : a.buq) + (size_t)g * a.nv;
+  return (cls < Q_BUL ? a.tdq : a.buq) + (size_t)g * a.nva;
 }
 // entry i of queue class cls (light classes from the front, heavy from the back)
 template <typename T>
 __device__ __forceinline__ uint32_t queue_at(const BatchArgs<T> &a, const uint32_t *q, int cls, uint32_t i) {
-  return (cls & 1) ? q[a.nv - 1 - i] : q[i];
+  return (cls & 1) ? q[a.nva - 1 - i] : q[i];
 }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -166,7 +171,7 @@ __device__ __forceinline__ void queue_push(const BatchArgs<T> &a, int g, uint32_
   if (pred) {
     const uint32_t i = base + __popc(bal & lanemask_lt());
     uint32_t *q = queue_of(a, g, cls);
-    if (cls & 1) q[a.nv - 1 - i] = v; else q[i] = v;
+    if (cls & 1) q[a.nva - 1 - i] = v; else q[i] = v;
   }
 }
 
@@ -175,49 +180,81 @@ __device__ __forceinline__ int queue_class(uint32_t d, bool bu) {
 }
 
 // ------------------------------------------------------------------------- init ----
-// Control words, per-level counters and the item counters (one CTA per group).
+// Control words, per-level counters and the item counters (one CTA per group).  Level 1
+// has closed-form Eq. 1 counters over all nv vertices (reading #23): top-down, the
+// frontier is the distinct sources (sum_j |FQ_j| = rows); bottom-up, every vertex but the
+// instance's own source is unvisited (sum_j |FQ_j| = rows * (nv - 1), |JFQ| = nv unless
+// every source is the same vertex).  Instances whose source is isolated are finished at
+// level 0: they are left out of the active mask, and a group of only such instances is
+// done before level 1 (its rows are -1 except the source).
 template <typename T>
 __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
+  constexpr int W = WordBits<T>::value;
+  __shared__ uint32_t s_src[W];
+  __shared__ uint32_t s_distinct;
+  __shared__ T s_act;
   const int g = blockIdx.x;
   const int rows = group_rows(a, g);
   LevelStat *ls = a.lstat + (size_t)g * MAXL;
   for (int l = threadIdx.x; l < MAXL; l += blockDim.x) ls[l] = LevelStat{};
+  if (threadIdx.x == 0) { s_distinct = 0; s_act = wzero_value<T>(); }
+  for (int j = threadIdx.x; j < rows; j += blockDim.x) s_src[j] = a.src[(size_t)g * W + j];
+  __syncthreads();
+  for (int j = threadIdx.x; j < rows; j += blockDim.x) {
+    bool first = true;
+    for (int i = 0; i < j; ++i)
+      if (s_src[i] == s_src[j]) { first = false; break; }
+    if (first) atomicAdd(&s_distinct, 1u);
+    if (a.csrc[(size_t)g * W + j] != NO_VERTEX) set_bit_atomic(&s_act, j);
+  }
+  __syncthreads();
   if (threadIdx.x == 0) {
     GroupCtrl<T> c;
-    c.active = wlowmask<T>(rows);
+    c.active = s_act;
     c.newacc = wzero_value<T>();
     c.n_f = c.m_f = c.newp = 0;
     for (int p = 0; p < 2; ++p)
       for (int k = 0; k < 4; ++k) c.qlen[p][k] = 0;
     c.dir = first_dir;
-    c.done = rows == 0 ? 1u : 0u;
+    const bool done = rows == 0 || wzero(s_act);
+    c.done = done ? 1u : 0u;
     c.arrive = 0;
-    c.last_level = 0;
-    c.iso_jfq1 = c.iso_fq1 = 0;
+    c.last_level = done ? 0xffffffffu : 0u;  // done at init: no snapshot was ever written
     a.ctrl[g] = c;
-    if (rows == 0) atomicAdd(a.batch_done, 1u);
+    if (rows > 0) {
+      LevelStat *l1 = ls + 1;
+      if (first_dir == 0) {
+        l1->jfq = s_distinct;
+        l1->fq = (unsigned long long)rows;
+      } else {
+        l1->jfq = (unsigned long long)a.nv - (s_distinct == 1 ? 1u : 0u);
+        l1->fq = (unsigned long long)rows * ((unsigned long long)a.nv - 1ull);
+      }
+      if (done) l1->dir = first_dir + 1;  // level 1 "runs" and finds nothing
+    }
+    if (done) atomicAdd(a.batch_done, 1u);
   }
   if (g == 0)
     for (int l = threadIdx.x; l < MAXL; l += blockDim.x) a.work_ctr[l] = 0;
 }
 
 // Zero the group's visited words and the snapshot slots of levels 0 and 1 (a2); when
-// level 1 runs bottom-up, enqueue every vertex of degree 1..HUB_T (all are unvisited
-// for some instance unless they are the source of every instance -- the expand skips
-// those).
+// level 1 runs bottom-up, enqueue every vertex of degree <= HUB_T (all are unvisited for
+// some active instance unless they are the source of every active instance -- the
+// expand skips those).
 template <typename T>
 __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint32_t first_dir) {
   const int g = blockIdx.y;
-  if (group_rows(a, g) == 0) return;
+  if (a.ctrl[g].done) return;
   const size_t stride = (size_t)gridDim.x * BLOCK;
   const T z = wzero_value<T>();
   T *vis = a.visited + (size_t)g * a.gstride;
   T *s0 = snap(a, g, 0);
   T *s1 = snap(a, g, 1);
   uint32_t *qlen = a.ctrl[g].qlen[0];
-  const size_t nvr = ((size_t)a.nv + 31) & ~(size_t)31;  // warp-uniform trip count
+  const size_t nvr = ((size_t)a.nva + 31) & ~(size_t)31;  // warp-uniform trip count
   for (size_t v = (size_t)blockIdx.x * BLOCK + threadIdx.x; v < nvr; v += stride) {
-    const bool in = v < a.nv;
+    const bool in = v < a.nva;
     if (in) {
       st(vis + v, z);
       st(s0 + v, z);
@@ -225,33 +262,31 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
     }
     if (first_dir) {
       const uint32_t d = in ? __ldg(a.deg + v) : 0u;
-      const bool q = d > 0 && d <= (uint32_t)HUB_T;
+      const bool q = in && d <= (uint32_t)HUB_T;
       queue_push(a, g, qlen, Q_BUL, q && d <= (uint32_t)LIGHT_DEG, (uint32_t)v);
       queue_push(a, g, qlen, Q_BUH, q && d > (uint32_t)LIGHT_DEG, (uint32_t)v);
     }
   }
 }
 
-// Sources: visited[s_j] |= bit j, S_0[s_j] |= bit j (depth 0); the distinct non-hub
-// source vertices form the top-down queue of level 1; level-1 statistics.
+// Sources: visited[s_j] |= bit j, S_0[s_j] |= bit j (depth 0) for the non-isolated
+// sources; the distinct ones of degree <= HUB_T form the top-down queue of level 1.
 template <typename T>
 __global__ void init_sources_kernel(BatchArgs<T> a, uint32_t first_dir) {
   constexpr int W = WordBits<T>::value;
   __shared__ uint32_t s_src[W];
-  __shared__ uint32_t s_cnt[3];
   const int g = blockIdx.x;
   const int rows = group_rows(a, g);
-  if (rows == 0) return;
+  if (rows == 0 || a.ctrl[g].done) return;
   T *vis = a.visited + (size_t)g * a.gstride;
   T *f = snap(a, g, 0);  // frontier of level 1
-  if (threadIdx.x < 3) s_cnt[threadIdx.x] = 0;
-  for (int j = threadIdx.x; j < rows; j += blockDim.x) s_src[j] = a.src[(size_t)g * W + j];
+  for (int j = threadIdx.x; j < rows; j += blockDim.x) s_src[j] = a.csrc[(size_t)g * W + j];
   __syncthreads();
   uint32_t *qlen = a.ctrl[g].qlen[0];
   for (int j = threadIdx.x; j < W; j += blockDim.x) {  // warp-uniform loop
     bool first = false;
     uint32_t s = 0, d = 0;
-    if (j < rows) {
+    if (j < rows && s_src[j] != NO_VERTEX) {
       s = s_src[j];
       set_bit_atomic(vis + s, j);
       set_bit_atomic(f + s, j);
@@ -259,26 +294,10 @@ __global__ void init_sources_kernel(BatchArgs<T> a, uint32_t first_dir) {
       for (int i = 0; i < j; ++i)
         if (s_src[i] == s) { first = false; break; }
       d = __ldg(a.deg + s);
-      if (first) atomicAdd(&s_cnt[0], 1u);          // distinct sources: |JFQ| of level 1
-      if (d == 0) atomicAdd(&s_cnt[1], 1u);         // rows whose source is isolated
     }
-    const bool q = first && d > 0 && d <= (uint32_t)HUB_T && first_dir == 0;
+    const bool q = first && d <= (uint32_t)HUB_T && first_dir == 0;
     queue_push(a, g, qlen, Q_TDL, q && d <= (uint32_t)LIGHT_DEG, s);
     queue_push(a, g, qlen, Q_TDH, q && d > (uint32_t)LIGHT_DEG, s);
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    LevelStat *ls = a.lstat + (size_t)g * MAXL + 1;
-    if (first_dir == 0) {
-      ls->jfq = s_cnt[0];
-      ls->fq = (unsigned long long)rows;
-    } else {
-      // bottom-up level 1, isolated vertices: T = active & ~(own source bits)
-      bool all_same_iso = __ldg(a.deg + s_src[0]) == 0;
-      for (int j = 1; j < rows && all_same_iso; ++j) all_same_iso = s_src[j] == s_src[0];
-      ls->jfq = (unsigned long long)a.n_iso - (all_same_iso ? 1u : 0u);
-      ls->fq = (unsigned long long)a.n_iso * rows - s_cnt[1];
-    }
   }
 }
 
@@ -481,7 +500,7 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       } else {
         const T tx = tx_next;
         const bool keep = !wzero(tx);
-        if (keep) { jfq++; fq += wpopc(tx); }
+        if (keep && level > 1) { jfq++; fq += wpopc(tx); }  // level 1: closed form (init)
         const uint32_t bal = __ballot_sync(FULL, keep);
         if (keep) {
           const uint32_t pos = qbase + ((tail + __popc(bal & lanemask_lt())) & (QW - 1));
@@ -613,7 +632,8 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
     }
     if (tid == 0 && !wzero(acc)) { red_or(N + c.v, acc); writes++; }
   }
-  flush_counts(sm, g, first ? 1u : 0u, first ? (uint32_t)wpopc(tg) : 0u, first ? 1u : 0u, insp, writes);
+  const bool cnt = first && level > 1;  // level 1: closed form (init)
+  flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tg) : 0u, first ? 1u : 0u, insp, writes);
 }
 
 // One launch per level for all groups of a batch.  Work items, pulled by CTAs from a
@@ -738,7 +758,7 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
   T *Z = snap(a, g, level + 1);  // target of the next level's expand
   T *vis = a.visited + (size_t)g * a.gstride;
   uint32_t *qlen = c->qlen[level & 1];
-  const size_t nv = a.nv;
+  const size_t nv = a.nva;
   unsigned long long nf = 0, mf = 0, newp = 0;
   T nacc = wzero_value<T>();
   const size_t stride = (size_t)gridDim.x * BLOCK;
@@ -884,17 +904,57 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
 // ------------------------------------------------------------------------ depth ----
 // Depth rows from the level snapshots l in [l0, l1] (l1 capped at the group's last
 // committed level and at 127): depth[j][v] = the first l with bit j of S_l[v] set.
-// One CTA handles DT consecutive vertices x all W rows: each thread (= one vertex)
-// accumulates (l + 1) into the byte of every row whose bit first appears at level l
-// (4 rows per 32-bit register, SIMD-within-a-register: bytes never carry since each
-// receives at most one value <= 128), stores its bytes into a [W][DT] shared tile, and
-// the CTA writes the tile row by row with full 128-byte lines.  first != 0 writes every
-// byte (-1 where no bit was found); otherwise only the bytes found in [l0, l1] change.
-constexpr int DT = 128;
+//
+// A CTA owns a tile of DV consecutive caller-id vertices (columns) x all W rows, staged
+// in a shared [W][DV] byte tile prefilled with -1 (isolated vertices own no snapshot
+// word).  The tile's vertices of degree > 0 are one contiguous range [c0, c0 + k) of
+// compacted ids, so each level's words for the tile are one contiguous run: thread 0
+// fetches them with 1-D TMA bulk copies (cp.async.bulk, DLB levels per stage, DNS stages
+// completing on mbarriers), DNS - 1 jobs ahead of the consumers, across tile boundaries.
+// Consumers are dealt densely over the k vertices (no lane idles on an isolated column):
+// thread t owns vertex slots t%64 and t%64 + 64 for the W/2 instances of half t/64,
+// and accumulates (l + 1) into the byte of every row whose bit first appears at level l
+// (SIMD within a register: bytes never carry, each receives at most one value <= 128).
+// An isolated source gets 0 in its own row.  The tile is written row by row with 16-byte
+// stores (full 128-byte lines).  first != 0 writes every byte; otherwise only the bytes
+// found in [l0, l1] change (a ring-slot flush before reuse).
+constexpr int DV = 128;         // columns per tile
+constexpr int DTHREADS = 128;
+constexpr int DLB = 4;          // levels per pipeline stage
+constexpr int DNS = 4;          // pipeline stages (DNS - 1 jobs in flight)
+constexpr int DSLOTS = DTHREADS / 2;  // vertex slots per pass (two halves per vertex)
+constexpr int DROWB = DV + 16;  // bytes per tile row (padded, 16-byte aligned)
 
 __device__ __forceinline__ uint32_t spread4(uint32_t nib) {
   // 4-bit nibble -> 0x01 in each byte whose bit is set
   return (nib * 0x00204081u) & 0x01010101u;
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(unsigned long long *bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// 1-D TMA bulk copy global -> shared (16-byte aligned, size a multiple of 16), completing
+// `bytes` of transaction count on the mbarrier.
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, unsigned long long *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
 }
 
 // m16n8k32 u8 x u8 -> s32 tensor-core MMA (D += A * B), fragments per the PTX ISA.
@@ -930,114 +990,249 @@ __device__ __forceinline__ void flush_macc(int (&dacc)[NT][4], unsigned long lon
   for (int nt = 0; nt < NT; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
 }
 
-// The same pass accumulates m_s (reading #11): every byte it finds adds deg(v) to row j's
-// sum (each (j, v) is found in exactly one flush) -- a [4 x DT] x [DT x W] u8 product per
-// tile on the tensor cores, flushed to m_out once per CTA.  CTAs loop over vertex tiles.
-constexpr int DTHREADS = DT;  // one thread per vertex of the tile
+template <typename T>
+struct DepthLayout {
+  static constexpr int W = WordBits<T>::value;
+  static constexpr size_t SROW = (size_t)DV * sizeof(T) + 16;  // one level's run (+ alignment slack)
+  static constexpr size_t TILE = (size_t)W * DROWB;
+  static constexpr size_t STAGE = DLB * SROW;
+  static constexpr size_t BYTES = TILE + DNS * STAGE;
+};
 
 template <typename T>
-__global__ void __launch_bounds__(DTHREADS) depth_kernel(BatchArgs<T> a, int l0, int l1, int first,
-                                                        unsigned long long *m_out) {
+constexpr size_t depth_smem_bytes() {
+  return DepthLayout<T>::BYTES;
+}
+
+__device__ __forceinline__ void mbar_arrive(unsigned long long *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+// barrier among the DTHREADS consumer threads only (the producer warp never joins)
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(DTHREADS) : "memory"); }
+
+// The same pass accumulates m_s (reading #11): every byte it finds adds deg(v) to row j's
+// sum (each (j, v) is found in exactly one flush) -- a [4 x DV] x [DV x W] u8 product per
+// tile on the tensor cores, flushed to m_out once per CTA.
+//
+// Warp roles: warps 0 .. DTHREADS/32 - 1 consume; the last warp produces (one lane issues
+// the bulk copies).  Stage st is "full" when its bytes landed (s_full[st], expect_tx) and
+// "empty" when every consumer warp has read it (s_empty[st], one arrive per warp).
+template <typename T>
+__global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a, int l0, int l1, int first,
+                                                                unsigned long long *m_out) {
+  using L = DepthLayout<T>;
   constexpr int W = WordBits<T>::value;
-  constexpr int Q = W / 4;  // 32-bit registers of depth bytes per vertex
-  constexpr int ROWW = DT / 4 + 1;
-  constexpr int ROWB = ROWW * 4;
-  constexpr int NWD = DTHREADS / 32;               // warps
+  constexpr int HQ = W / 8;                        // 32-bit byte registers per (vertex, half)
+  constexpr int NWD = DTHREADS / 32;               // consumer warps
   constexpr int NTILES = W / 8;                    // 8-row n-tiles of the MMA
   constexpr int NTW = NTILES >= NWD ? NTILES / NWD : 1;
   constexpr int MMA_WARPS = NTILES / NTW;          // warps taking part in the MMA
-  __shared__ __align__(16) uint32_t tile[W][ROWW];
-  __shared__ uint32_t s_deg[DT];
+  extern __shared__ __align__(128) unsigned char dsm[];
+  unsigned char *tb = dsm;                          // [W][DROWB]
+  unsigned char *stage_base = dsm + L::TILE;        // [DNS][DLB][SROW]
+  __shared__ __align__(8) unsigned long long s_full[DNS], s_empty[DNS];
+  __shared__ uint32_t s_deg[DV];
+  __shared__ uint16_t s_col[DV];
+  __shared__ uint32_t s_wcnt[NWD];
   __shared__ unsigned long long s_m[W];
+  __shared__ uint32_t s_isrc[W];  // caller id of row j's source if it is isolated, else NO_VERTEX
+  __shared__ uint32_t s_has_iso;
+  __shared__ uint32_t s_stage_off[DNS];  // byte offset of element 0 inside each stage row
   const int g = blockIdx.y;
   const int rows = group_rows(a, g);
   if (rows == 0) return;
   const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
   const int gq = lane >> 2, tq4 = lane & 3;  // mma fragment coordinates
-  int dacc[NTW][4];
-#pragma unroll
-  for (int nt = 0; nt < NTW; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
-  int tiles_acc = 0;
-  for (int j = t; j < W; j += DTHREADS) s_m[j] = 0;
+  const int slot = t % DSLOTS, half = t / DSLOTS;
   const GroupCtrl<T> *c = a.ctrl + g;
   const int last = min((int)c->last_level, min(l1, 127));
+  const int nlev = last - l0 + 1;  // levels to read (may be <= 0)
+  const int nbat = nlev > 0 ? (nlev + DLB - 1) / DLB : 0;
   int8_t *out = a.out + (size_t)g * W * a.nv;
   const size_t nvv = a.nv;
-  const size_t ntiles = (nvv + DT - 1) / DT;
-  unsigned char *tb = reinterpret_cast<unsigned char *>(&tile[0][0]);
-  const int8_t *tile_bytes = reinterpret_cast<const int8_t *>(tb);
-  for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x) {
-    const size_t v0 = tix * DT;
-    const size_t v = v0 + t;
-    const bool in = v < nvv;
-    uint32_t acc[Q];
-#pragma unroll
-    for (int q = 0; q < Q; ++q) acc[q] = 0;
-    if (in) {
-      T reached = wzero_value<T>();
-      for (int l = l0; l <= last; ++l) {
-        const T nb = wandn(ld(snap(a, g, l) + v), reached);
-        if (wzero(nb)) continue;
-        reached = wor(reached, nb);
-        const uint32_t inc = (uint32_t)(l + 1);
-#pragma unroll
-        for (int q = 0; q < Q; ++q) {
-          const uint32_t nib = (wpiece(nb, q >> 3) >> ((q & 7) * 4)) & 0xFu;
-          acc[q] += spread4(nib) * inc;
-        }
-      }
+  const size_t ntiles = (nvv + DV - 1) / DV;
+  const size_t ntb = (nvv + 127) / 128;  // entries of tbase - 1
+  const size_t my_tiles = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+  const size_t njobs = my_tiles * (size_t)nbat;
+  if (t == 0) {
+    s_has_iso = 0;
+    for (int k = 0; k < DNS; ++k) {
+      mbar_init(&s_full[k], 1);
+      mbar_init(&s_empty[k], NWD);
     }
-    __syncthreads();  // previous tile fully written out
-    s_deg[t] = in ? __ldg(a.deg + v) : 0u;
-#pragma unroll
-    for (int q = 0; q < Q; ++q) {
-      const uint32_t x = __vsub4(acc[q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
-#pragma unroll
-      for (int b = 0; b < 4; ++b) tb[(q * 4 + b) * ROWB + t] = (unsigned char)(x >> (8 * b));
-    }
-    __syncthreads();
-    // m_s on the tensor cores: D[b][j] += sum_v deg_b(v) * reached(j, v), deg_b = byte b
-    // of deg(v) (A: 16 x 32 u8, rows 0..3 = byte planes), reached from the tile (B: 32 x 8
-    // u8, 0/1); m_s[j] = sum_b D[b][j] << 8b.
-    if (warp < MMA_WARPS) {
-#pragma unroll
-      for (int ks = 0; ks < DT / 32; ++ks) {
-        uint32_t a0 = 0, a2 = 0;
-        if (gq < 4) {
-          const int vb = ks * 32 + tq4 * 4;
-          a0 = byte_plane4(s_deg + vb, gq);
-          a2 = byte_plane4(s_deg + vb + 16, gq);
-        }
-#pragma unroll
-        for (int nt = 0; nt < NTW; ++nt) {
-          const int j = (warp * NTW + nt) * 8 + gq;
-          const uint32_t b0 = __vcmpne4(tile[j][ks * 8 + tq4], 0xffffffffu) & 0x01010101u;
-          const uint32_t b1 = __vcmpne4(tile[j][ks * 8 + 4 + tq4], 0xffffffffu) & 0x01010101u;
-          mma_u8_m16n8k32(dacc[nt], a0, 0u, a2, 0u, b0, b1);
-        }
-      }
-      if (++tiles_acc == 4096) {  // int32 headroom: <= 4 * 32 * 255 per tile and element
-        flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
-        tiles_acc = 0;
-      }
-    }
-    const bool vec = first && ((nvv & 15) == 0) && (((uintptr_t)out & 15) == 0) && (v0 + DT <= nvv);
-    if (vec) {
-      // 8 threads x 16 bytes per 128-byte row segment; DTHREADS/8 rows per pass
-      const int sub = t & 7, r0 = t >> 3;
-      for (int j = r0; j < rows; j += DTHREADS / 8) {
-        const uint32_t *src = &tile[j][sub * 4];
-        *reinterpret_cast<int4 *>(out + (size_t)j * nvv + v0 + sub * 16) =
-            make_int4((int)src[0], (int)src[1], (int)src[2], (int)src[3]);
-      }
-    } else if (v < nvv) {
-      for (int j = 0; j < rows; ++j) {
-        const int8_t d = tile_bytes[j * ROWB + t];
-        if (first || d != -1) out[(size_t)j * nvv + v] = d;
-      }
-    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp < MMA_WARPS) flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
+  __syncthreads();
+  if (warp == NWD) {
+    // ---- producer: job jb = (tile jb / nbat of this CTA, batch jb % nbat) -> stage jb % DNS
+    if (lane == 0 && njobs) {
+      uint32_t c0n = __ldg(a.tbase + blockIdx.x * (DV / 128));
+      uint32_t c1n = __ldg(a.tbase + min((size_t)blockIdx.x * (DV / 128) + DV / 128, ntb));
+      uint32_t c0 = 0, k = 0;
+      for (size_t jb = 0; jb < njobs; ++jb) {
+        const int st = (int)(jb % DNS);
+        const int b = (int)(jb % nbat);
+        if (b == 0) {  // a new tile: take its prefetched range, prefetch the next tile's
+          c0 = c0n;
+          k = c1n - c0n;
+          const size_t nt = blockIdx.x + (jb / nbat + 1) * gridDim.x;
+          if (nt < ntiles) {
+            c0n = __ldg(a.tbase + nt * (DV / 128));
+            c1n = __ldg(a.tbase + min(nt * (DV / 128) + DV / 128, ntb));
+          }
+        }
+        if (jb >= (size_t)DNS) mbar_wait(&s_empty[st], (uint32_t)((jb / DNS - 1) & 1));
+        const int lb = l0 + b * DLB, le = min(last, lb + DLB - 1);
+        uint32_t total = 0, off = 0, size = 0;
+        if (k) {
+          const uintptr_t src0 = (uintptr_t)(snap(a, g, lb) + c0);
+          off = (uint32_t)(src0 & 15u);
+          size = (uint32_t)((off + (size_t)k * sizeof(T) + 15) & ~(size_t)15);
+          total = size * (uint32_t)(le - lb + 1);
+        }
+        s_stage_off[st] = off;
+        mbar_arrive_expect_tx(&s_full[st], total);
+        if (k)
+          for (int l = lb; l <= le; ++l) {
+            const unsigned char *src = reinterpret_cast<const unsigned char *>(snap(a, g, l) + c0) - off;
+            bulk_g2s(stage_base + (size_t)st * L::STAGE + (size_t)(l - lb) * L::SROW, src, size, &s_full[st]);
+          }
+      }
+    }
+  } else {
+    // ---- consumers
+    const uint32_t *tw = reinterpret_cast<const uint32_t *>(tb);
+    int dacc[NTW][4];
+#pragma unroll
+    for (int nt = 0; nt < NTW; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
+    int tiles_acc = 0;
+    for (int j = t; j < W; j += DTHREADS) {
+      s_m[j] = 0;
+      uint32_t x = NO_VERTEX;
+      if (j < rows && a.csrc[(size_t)g * W + j] == NO_VERTEX) {
+        x = a.src[(size_t)g * W + j];
+        s_has_iso = 1;
+      }
+      s_isrc[j] = x;
+    }
+    size_t job = 0;
+    for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x) {
+      const size_t v0 = tix * DV;
+      const size_t v = v0 + t;
+      // ranks of the non-isolated columns; prefill -1 (the previous tile is written out)
+      const uint32_t word = v < nvv ? __ldg(a.nzbits + (v >> 5)) : 0u;
+      const bool nz = (word >> lane) & 1u;
+      const uint32_t c0t = __ldg(a.tbase + tix * (DV / 128));
+      if (lane == 0) s_wcnt[warp] = __popc(word);
+      s_deg[t] = 0;
+      for (int k4 = t; k4 < (int)(L::TILE / 16); k4 += DTHREADS)
+        reinterpret_cast<int4 *>(tb)[k4] = make_int4(-1, -1, -1, -1);
+      consumers_sync();
+      uint32_t before = 0, kcount = 0;
+#pragma unroll
+      for (int w = 0; w < NWD; ++w) {
+        const uint32_t x = s_wcnt[w];
+        before += w < warp ? x : 0u;
+        kcount += x;
+      }
+      if (nz) s_col[before + __popc(word & ((1u << lane) - 1u))] = (uint16_t)t;
+      uint32_t acc[2][HQ];
+#pragma unroll
+      for (int r = 0; r < 2; ++r)
+#pragma unroll
+        for (int q = 0; q < HQ; ++q) acc[r][q] = 0;
+      unsigned long long reached[2] = {0ull, 0ull};
+      for (int b = 0; b < nbat; ++b, ++job) {
+        const int st = (int)(job % DNS);
+        mbar_wait(&s_full[st], (uint32_t)((job / DNS) & 1));
+        const unsigned char *sb = stage_base + (size_t)st * L::STAGE + s_stage_off[st];
+        const int lb = l0 + b * DLB, le = min(last, lb + DLB - 1);
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+          const uint32_t i = slot + DSLOTS * r;
+          if (i < kcount) {
+#pragma unroll
+            for (int u = 0; u < DLB; ++u) {
+              if (lb + u > le) break;
+              const T wv = *reinterpret_cast<const T *>(sb + (size_t)u * L::SROW + (size_t)i * sizeof(T));
+              const unsigned long long hb = whalf(wv, half) & ~reached[r];
+              if (!hb) continue;
+              reached[r] |= hb;
+              const uint32_t inc = (uint32_t)(lb + u + 1);
+#pragma unroll
+              for (int q = 0; q < HQ; ++q) acc[r][q] += spread4((uint32_t)(hb >> (4 * q)) & 0xFu) * inc;
+            }
+          }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&s_empty[st]);  // this warp is done with stage st
+      }
+      // the tile's columns
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const uint32_t i = slot + DSLOTS * r;
+        if (i < kcount) {
+          const int col = s_col[i];
+          if (half == 0) s_deg[col] = __ldg(a.deg + c0t + i);
+#pragma unroll
+          for (int q = 0; q < HQ; ++q) {
+            const uint32_t x = __vsub4(acc[r][q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
+#pragma unroll
+            for (int bb = 0; bb < 4; ++bb)
+              tb[(half * (W / 2) + q * 4 + bb) * DROWB + col] = (unsigned char)(x >> (8 * bb));
+          }
+        }
+      }
+      consumers_sync();
+      if (s_has_iso) {  // isolated sources: depth 0 in their own row (degree 0: no m_s)
+        for (int j = t; j < rows; j += DTHREADS) {
+          const uint32_t s = s_isrc[j];
+          if (s != NO_VERTEX && s >= v0 && s < v0 + DV) tb[j * DROWB + (s - v0)] = 0;
+        }
+        consumers_sync();
+      }
+      // m_s on the tensor cores: D[b][j] += sum_v deg_b(v) * reached(j, v), deg_b = byte b
+      // of deg(v) (A: 16 x 32 u8, rows 0..3 = byte planes), reached from the tile (B: 32 x
+      // 8 u8, 0/1); m_s[j] = sum_b D[b][j] << 8b.
+      if (kcount && warp < MMA_WARPS) {
+#pragma unroll
+        for (int ks = 0; ks < DV / 32; ++ks) {
+          uint32_t a0 = 0, a2 = 0;
+          if (gq < 4) {
+            const int vb = ks * 32 + tq4 * 4;
+            a0 = byte_plane4(s_deg + vb, gq);
+            a2 = byte_plane4(s_deg + vb + 16, gq);
+          }
+#pragma unroll
+          for (int nt = 0; nt < NTW; ++nt) {
+            const int j = (warp * NTW + nt) * 8 + gq;
+            const uint32_t b0 = __vcmpne4(tw[j * (DROWB / 4) + ks * 8 + tq4], 0xffffffffu) & 0x01010101u;
+            const uint32_t b1 = __vcmpne4(tw[j * (DROWB / 4) + ks * 8 + 4 + tq4], 0xffffffffu) & 0x01010101u;
+            mma_u8_m16n8k32(dacc[nt], a0, 0u, a2, 0u, b0, b1);
+          }
+        }
+        if (++tiles_acc == 4096) {  // int32 headroom: <= DV * 255 per tile and element
+          flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
+          tiles_acc = 0;
+        }
+      }
+      const bool vec = first && ((nvv & 15) == 0) && (((uintptr_t)out & 15) == 0) && (v0 + DV <= nvv);
+      if (vec) {
+        // DV/16 threads x 16 bytes per row segment; DTHREADS/(DV/16) rows per pass
+        const int sub = t % (DV / 16), r0 = t / (DV / 16);
+        for (int j = r0; j < rows; j += DTHREADS / (DV / 16))
+          *reinterpret_cast<int4 *>(out + (size_t)j * nvv + v0 + sub * 16) =
+              *reinterpret_cast<const int4 *>(tb + j * DROWB + sub * 16);
+      } else if (v < nvv) {
+        for (int j = 0; j < rows; ++j) {
+          const int8_t d = (int8_t)tb[j * DROWB + t];
+          if (first || d != -1) out[(size_t)j * nvv + v] = d;
+        }
+      }
+      consumers_sync();  // tile and s_deg / s_col reused by the next tile
+    }
+    if (warp < MMA_WARPS) flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
+  }
   __syncthreads();
   for (int j = t; j < rows; j += DTHREADS)
     if (s_m[j]) atomicAdd(&m_out[(size_t)g * W + j], s_m[j]);

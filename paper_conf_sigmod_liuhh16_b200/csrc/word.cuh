@@ -58,6 +58,13 @@ __device__ __forceinline__ uint32_t wpiece(u128 a, int k) {
   return (uint32_t)(h >> (32 * (k & 1)));
 }
 
+// Bits [h * W/2, (h + 1) * W/2) of a word, h in {0, 1}, right-aligned.
+__device__ __forceinline__ unsigned long long whalf(uint32_t a, int h) { return h ? (a >> 16) : (a & 0xffffu); }
+__device__ __forceinline__ unsigned long long whalf(unsigned long long a, int h) {
+  return h ? (a >> 32) : (a & 0xffffffffull);
+}
+__device__ __forceinline__ unsigned long long whalf(u128 a, int h) { return h ? a.hi : a.lo; }
+
 // word with the low `n` bits set (n <= W): the real instances of a (possibly short) group
 template <typename T> __host__ __device__ __forceinline__ T wlowmask(int n);
 template <> __host__ __device__ __forceinline__ uint32_t wlowmask<uint32_t>(int n) {

@@ -178,6 +178,9 @@ struct ibfs_graph {
   uint32_t *d_nzbits = nullptr;         // [nv/32]: bit v%32 of word v/32 = (deg(v) > 0)
   HubChunk *d_chunks = nullptr;
   uint32_t n_chunks = 0;
+  uint32_t *d_hub_vtx = nullptr;     // [n_hubs] vertices of degree > HUB_T (ascending)
+  uint32_t *d_hub_chunk0 = nullptr;  // [n_hubs + 1] first chunk of each hub
+  uint32_t n_hubs = 0;
   std::vector<uint64_t> h_off;      // host copy of d_off (tiling, planner)
   std::vector<uint32_t> h_tbase, h_nzbits;
   int num_sms = 148;
@@ -194,6 +197,8 @@ void graph_release(ibfs_graph *g) {
   cudaFree(g->d_adj);
   cudaFree(g->d_deg);
   cudaFree(g->d_chunks);
+  cudaFree(g->d_hub_vtx);
+  cudaFree(g->d_hub_chunk0);
   cudaFree(g->d_tbase);
   cudaFree(g->d_nzbits);
   if (prev >= 0) cudaSetDevice(prev);
@@ -272,7 +277,10 @@ __global__ void remap_adj_kernel(uint32_t *adj, unsigned long long ne, const uin
 void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig) {
   const uint32_t nv = g->nv;
   const uint32_t nwords = (nv + 31) / 32, ntiles = (nv + 127) / 128;
-  CK(cudaMalloc(&g->d_nzbits, std::max<size_t>(nwords, 1) * 4));
+  // padded to whole 128-vertex tiles (+1) so a tile's 4 words load as one uint4
+  const size_t nz_alloc = ((size_t)ntiles + 1) * 4;
+  CK(cudaMalloc(&g->d_nzbits, nz_alloc * 4));
+  CK(cudaMemset(g->d_nzbits, 0, nz_alloc * 4));
   CK(cudaMalloc(&g->d_tbase, ((size_t)ntiles + 1) * 4));
   uint32_t *cnt = nullptr;
   void *tmp = nullptr;
@@ -325,9 +333,12 @@ uint32_t host_compact_id(const ibfs_graph *g, uint32_t v) {
 // cut into chunks of CHUNK edges, each a work item a whole CTA sweeps.
 void build_decomposition(ibfs_graph *g) {
   std::vector<HubChunk> chunks;
+  std::vector<uint32_t> hubs, chunk0;
   for (uint32_t v = 0; v < g->nva; ++v) {
     const uint64_t d = g->h_off[v + 1] - g->h_off[v];
     if (d <= (uint64_t)HUB_T) continue;
+    hubs.push_back(v);
+    chunk0.push_back((uint32_t)chunks.size());
     uint32_t first = 1;
     for (uint64_t e = g->h_off[v]; e < g->h_off[v + 1]; e += CHUNK) {
       HubChunk c;
@@ -340,9 +351,15 @@ void build_decomposition(ibfs_graph *g) {
     }
   }
   g->n_chunks = (uint32_t)chunks.size();
+  chunk0.push_back(g->n_chunks);
+  g->n_hubs = (uint32_t)hubs.size();
   CK(cudaMalloc(&g->d_chunks, std::max<size_t>(chunks.size(), 1) * sizeof(HubChunk)));
   if (!chunks.empty())
     CK(cudaMemcpy(g->d_chunks, chunks.data(), chunks.size() * sizeof(HubChunk), cudaMemcpyHostToDevice));
+  CK(cudaMalloc(&g->d_hub_vtx, std::max<size_t>(hubs.size(), 1) * 4));
+  CK(cudaMalloc(&g->d_hub_chunk0, chunk0.size() * 4));
+  if (!hubs.empty()) CK(cudaMemcpy(g->d_hub_vtx, hubs.data(), hubs.size() * 4, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_hub_chunk0, chunk0.data(), chunk0.size() * 4, cudaMemcpyHostToDevice));
 }
 
 // Degrees, max degree, hub chunks; compacted offsets must be in g->d_off and g->h_off.
@@ -767,6 +784,39 @@ namespace {
 
 constexpr int LEVELS_PER_CHECK = 2;
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda needed).
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_tiled_fn() {
+  static EncodeTiledFn fn = [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+    }
+    return reinterpret_cast<EncodeTiledFn>(p);
+  }();
+  return fn;
+}
+
+// [rows][nv] int8 rows at `base` (row stride nv bytes) as a 2-D tensor with [W][DV] boxes,
+// 128-byte swizzle (the depth kernel's shared tile layout).  false if unavailable.
+bool encode_rows_map(CUtensorMap *map, void *base, uint32_t nv, uint32_t rows, int W) {
+  EncodeTiledFn fn = encode_tiled_fn();
+  if (!fn || rows == 0) return false;
+  const cuuint64_t dims[2] = {nv, rows};
+  const cuuint64_t strides[1] = {nv};
+  const cuuint32_t box[2] = {(cuuint32_t)DV, (cuuint32_t)W};
+  const cuuint32_t estr[2] = {1, 1};
+  return fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 // Per-thread, per-device cache of CUDA events and a pinned host word buffer: creating
 // them per call (cudaEventCreate, cudaMallocHost) costs far more than a small level.
 struct DevCache {
@@ -850,6 +900,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   T *ring = sc.get<T>((size_t)R * G * gstride);
   uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
+  uint32_t *chq = sc.get<uint32_t>((size_t)G * 2 * std::max<uint32_t>(g->n_chunks, 1));
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
   LevelStat *lstat = sc.get<LevelStat>((size_t)G * MAXL);
   uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
@@ -886,6 +937,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.n_total = n;
   a.chunks = g->d_chunks;
   a.n_chunks = g->n_chunks;
+  a.hub_vtx = g->d_hub_vtx;
+  a.hub_chunk0 = g->d_hub_chunk0;
+  a.n_hubs = g->n_hubs;
+  a.chq = chq;
   a.tdq = tdq;
   a.buq = buq;
   a.n_iso = nv - nva;
@@ -939,12 +994,19 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         1, std::min<uint64_t>(((uint64_t)nva + BLOCK * 4 - 1) / (BLOCK * 4), (uint64_t)g->num_sms * 8 / Gb));
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
+    // the rows of this batch as a [rows_in_batch][nv] byte tensor for the depth kernel's TMA
+    // stores (first flush, 16-byte aligned rows); otherwise it writes bytes itself
+    CUtensorMap out_map;
+    std::memset(&out_map, 0, sizeof(out_map));
+    const bool tma_ok = (nv % 16 == 0) && (((uintptr_t)a.out & 15) == 0) && encode_rows_map(&out_map, a.out, nv, rows_in_batch, W);
     auto flush = [&](int l1) {
       cudaEvent_t d0 = nullptr, d1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
                                                                          std::max<uint64_t>(1, (uint64_t)g->num_sms * 3 / Gb)));
-      depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, flushed < 0 ? 1 : 0, d_m);
+      const int first = flushed < 0 ? 1 : 0;
+      depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(
+          a, flushed + 1, l1, first, d_m, out_map, (first && tma_ok) ? 1 : 0);
       if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
       launches++;
       st.depth_launches++;

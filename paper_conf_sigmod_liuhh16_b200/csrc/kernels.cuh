@@ -31,6 +31,7 @@
 // frontier's adjacency used by all instances, as CTA-cooperative expansion).
 #pragma once
 #include <cstdint>
+#include <cuda.h>
 #include "word.cuh"
 
 namespace ibfs {
@@ -52,6 +53,8 @@ constexpr unsigned FULL = 0xffffffffu;
 
 // queue classes
 constexpr int Q_TDL = 0, Q_TDH = 1, Q_BUL = 2, Q_BUH = 3;
+constexpr int Q_TDC = 4, Q_BUC = 5;  // hub-chunk queues (chunk indices, not vertices)
+constexpr int NQ = 6;
 
 struct HubChunk {
   unsigned long long e0, e1;
@@ -70,8 +73,10 @@ struct GroupCtrl {
   T active;   // instances that discovered something at the last committed level
   T newacc;   // OR of the new bits of the running commit
   unsigned long long n_f, m_f, newp;
-  uint32_t qlen[2][4];  // [parity of the producing level][queue class]
+  unsigned long long vpairs;  // (instance, vertex) pairs visited so far
+  uint32_t qlen[2][NQ]; // [parity of the producing level][queue class]
   uint32_t dir;         // direction of the next expand: 0 TD, 1 BU
+  uint32_t td_filter;   // top-down reads visited[w] before its RED.OR (else the commit masks)
   uint32_t done;
   uint32_t arrive;
   uint32_t last_level;
@@ -115,6 +120,10 @@ struct BatchArgs {
   int8_t *out;          // row g*W + j of this batch at out + (g*W + j) * nv
   const HubChunk *chunks;
   uint32_t n_chunks;
+  const uint32_t *hub_vtx;     // [n_hubs] compacted ids of the vertices of degree > HUB_T, ascending
+  const uint32_t *hub_chunk0;  // [n_hubs + 1] first chunk of each hub (chunks are in hub order)
+  uint32_t n_hubs;
+  uint32_t *chq;               // [gcap][2][n_chunks] hub-chunk queues (TD, BU)
   uint32_t n_iso;       // vertices of degree 0 (nv - nva)
   Policy pol;
 };
@@ -175,6 +184,39 @@ __device__ __forceinline__ void queue_push(const BatchArgs<T> &a, int g, uint32_
   }
 }
 
+// Enqueue every chunk of hub vertex v (degree > HUB_T) into hub-chunk queue cls (Q_TDC /
+// Q_BUC) when pred holds: the hub is a frontier of the next level, so its row is swept
+// chunk by chunk.  Warp-cooperative (all lanes must call it): the lanes holding a hub are
+// served one after the other, the whole warp writing each hub's chunk indices.
+template <typename T>
+__device__ __forceinline__ void push_hub_chunks(const BatchArgs<T> &a, int g, uint32_t *qlen, int cls,
+                                                bool pred, uint32_t v) {
+  uint32_t bal = __ballot_sync(FULL, pred);
+  if (!bal) return;
+  const int lane = threadIdx.x & 31;
+  uint32_t *q = a.chq + ((size_t)g * 2 + (cls - Q_TDC)) * a.n_chunks;
+  while (bal) {
+    const int src = __ffs(bal) - 1;
+    bal &= bal - 1;
+    const uint32_t hv = __shfl_sync(FULL, v, src);
+    uint32_t c0 = 0, c1 = 0, base = 0;
+    if (lane == 0) {
+      uint32_t lo = 0, hi = a.n_hubs;  // hub index: binary search (hubs are few and sorted)
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (__ldg(a.hub_vtx + mid) <= hv) lo = mid; else hi = mid;
+      }
+      c0 = __ldg(a.hub_chunk0 + lo);
+      c1 = __ldg(a.hub_chunk0 + lo + 1);
+      base = atomicAdd(qlen + cls, c1 - c0);
+    }
+    c0 = __shfl_sync(FULL, c0, 0);
+    c1 = __shfl_sync(FULL, c1, 0);
+    base = __shfl_sync(FULL, base, 0);
+    for (uint32_t c = c0 + lane; c < c1; c += 32) q[base + (c - c0)] = c;
+  }
+}
+
 __device__ __forceinline__ int queue_class(uint32_t d, bool bu) {
   return (bu ? Q_BUL : Q_TDL) + (d > (uint32_t)LIGHT_DEG ? 1 : 0);
 }
@@ -213,9 +255,11 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     c.active = s_act;
     c.newacc = wzero_value<T>();
     c.n_f = c.m_f = c.newp = 0;
+    c.vpairs = (unsigned long long)wpopc(s_act);
     for (int p = 0; p < 2; ++p)
-      for (int k = 0; k < 4; ++k) c.qlen[p][k] = 0;
+      for (int k = 0; k < NQ; ++k) c.qlen[p][k] = 0;
     c.dir = first_dir;
+    c.td_filter = 0;
     const bool done = rows == 0 || wzero(s_act);
     c.done = done ? 1u : 0u;
     c.arrive = 0;
@@ -265,6 +309,7 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
       const bool q = in && d <= (uint32_t)HUB_T;
       queue_push(a, g, qlen, Q_BUL, q && d <= (uint32_t)LIGHT_DEG, (uint32_t)v);
       queue_push(a, g, qlen, Q_BUH, q && d > (uint32_t)LIGHT_DEG, (uint32_t)v);
+      push_hub_chunks(a, g, qlen, Q_BUC, in && d > (uint32_t)HUB_T, (uint32_t)v);
     }
   }
 }
@@ -298,6 +343,7 @@ __global__ void init_sources_kernel(BatchArgs<T> a, uint32_t first_dir) {
     const bool q = first && d <= (uint32_t)HUB_T && first_dir == 0;
     queue_push(a, g, qlen, Q_TDL, q && d <= (uint32_t)LIGHT_DEG, s);
     queue_push(a, g, qlen, Q_TDH, q && d > (uint32_t)LIGHT_DEG, s);
+    push_hub_chunks(a, g, qlen, Q_TDC, first && d > (uint32_t)HUB_T && first_dir == 0, s);
   }
 }
 
@@ -399,6 +445,7 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
   const T *F = frontier_buf(a, g, level);
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
+  const bool filt = a.ctrl[g].td_filter != 0;
   const uint32_t *q = queue_of(a, g, cls);
   const uint32_t qn = i1 - i0;
   uint32_t insp = 0, writes = 0;
@@ -429,7 +476,7 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
     for (int u = 0; u < U; ++u) {
       if (w[u] != 0xffffffffu) {
         insp++;
-        const T b = wandn(fw[u], ldg(vis + w[u]));
+        const T b = filt ? wandn(fw[u], ldg(vis + w[u])) : fw[u];
         if (!wzero(b)) { red_or(N + w[u], b); writes++; }
       }
     }
@@ -570,6 +617,7 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
   const T *vis = a.visited + (size_t)g * a.gstride;
   const T f = ldg(F + c.v);
   if (wzero(f)) return;
+  const bool filt = a.ctrl[g].td_filter != 0;
   uint32_t insp = 0, writes = 0;
   constexpr int U = 8;
   for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
@@ -583,7 +631,7 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
     for (int u = 0; u < U; ++u) {
       if (w[u] != 0xffffffffu) {
         insp++;
-        const T b = wandn(f, ldg(vis + w[u]));
+        const T b = filt ? wandn(f, ldg(vis + w[u])) : f;
         if (!wzero(b)) { red_or(N + w[u], b); writes++; }
       }
     }
@@ -650,23 +698,26 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) expand_kernel(BatchAr
   for (int i = tid; i < a.G * 5; i += BLOCK) sm.acc[i / 5][i % 5] = 0ull;
   const int par = (level - 1) & 1;  // queues were produced by commit l-1 (or init)
   if (tid == 0) {
-    uint32_t ph = 0, pl = 0;
+    uint32_t ph = 0, pl = 0, pc = 0;
     for (int g = 0; g < a.G; ++g) {
       const GroupCtrl<T> &c = a.ctrl[g];
       sm.nitems[0][g] = ph;
       sm.nitems[1][g] = pl;
+      sm.nitems[2][g] = pc;
       if (!c.done) {
         const int base = c.dir ? Q_BUL : Q_TDL;
         const uint32_t qh = c.dir ? QBH : QH;
         ph += (c.qlen[par][base + 1] + qh - 1) / qh;
         pl += (c.qlen[par][base] + QL - 1) / QL;
+        pc += c.qlen[par][c.dir ? Q_BUC : Q_TDC];
       }
     }
     sm.nitems[0][a.G] = ph;
     sm.nitems[1][a.G] = pl;
+    sm.nitems[2][a.G] = pc;
   }
   __syncthreads();
-  const uint32_t n_hub = a.n_chunks * (uint32_t)a.G;
+  const uint32_t n_hub = sm.nitems[2][a.G];
   const uint32_t n_heavy = sm.nitems[0][a.G];
   const uint32_t total = n_hub + n_heavy + sm.nitems[1][a.G];
   uint32_t pending = 0;
@@ -681,10 +732,11 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) expand_kernel(BatchAr
     const uint32_t item = sm.item;
     if (item >= total) break;
     if (item < n_hub) {
-      const int g = (int)(item % (uint32_t)a.G);
+      int g = 0;
+      while (g + 1 < a.G && sm.nitems[2][g + 1] <= item) ++g;
       const GroupCtrl<T> *c = a.ctrl + g;
-      if (c->done) continue;
-      const HubChunk hc = a.chunks[item / (uint32_t)a.G];
+      const uint32_t k = item - sm.nitems[2][g];
+      const HubChunk hc = a.chunks[a.chq[((size_t)g * 2 + (c->dir ? 1 : 0)) * a.n_chunks + k]];
       if (c->dir == 0) hub_td<T>(a, sm, g, hc, level);
       else hub_bu<T>(a, sm, s_red, g, hc, level, c->active);
       continue;
@@ -775,7 +827,6 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
       vv[k] = wzero_value<T>();
       dg[k] = 0;
       if (v < nv) {
-        // S_l is disjoint from visited: TD masked it with the committed words, BU with T.
         n[k] = ld(N + v);
         vv[k] = ld(vis + v);
         dg[k] = __ldg(a.deg + v);
@@ -788,6 +839,11 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
       const size_t v = base + (size_t)k * BLOCK + tid;
       const bool in = v < nv;
       if (in) st(Z + v, wzero_value<T>());
+      {  // an unfiltered top-down level may have ORed already-visited bits: mask them
+        const T m = wandn(n[k], vv[k]);
+        if (in && !weq(m, n[k])) st(const_cast<T *>(N) + v, m);
+        n[k] = m;
+      }
       const bool nz = !wzero(n[k]);
       if (nz) st(vis + v, wor(vv[k], n[k]));
       const T tp = in ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
@@ -805,6 +861,9 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
       bal[k][Q_TDH] = __ballot_sync(FULL, nz && qd && !light);
       bal[k][Q_BUL] = __ballot_sync(FULL, un && qd && light);
       bal[k][Q_BUH] = __ballot_sync(FULL, un && qd && !light);
+      // hubs: their chunks, never the vertex queues
+      push_hub_chunks(a, g, qlen, Q_TDC, in && nz && d > (uint32_t)HUB_T, (uint32_t)v);
+      push_hub_chunks(a, g, qlen, Q_BUC, in && un && d > (uint32_t)HUB_T, (uint32_t)v);
 #pragma unroll
       for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
     }
@@ -878,9 +937,14 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
     c->newacc = wzero_value<T>();
     c->n_f = c->m_f = c->newp = 0;
     c->dir = bu ? 1u : 0u;
+    // top-down pre-check of visited[w] only once a fair share of the (vertex, active
+    // instance) pairs is visited; before that nearly every OR is new and the gather is
+    // wasted (the commit masks what an unfiltered OR set twice)
+    c->vpairs += np;
+    c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
     c->last_level = (uint32_t)level;
-    for (int k = 0; k < 4; ++k) c->qlen[(level + 1) & 1][k] = 0;  // target of commit l+1
+    for (int k = 0; k < NQ; ++k) c->qlen[(level + 1) & 1][k] = 0;  // target of commit l+1
     if (wzero(act)) {
       c->done = 1;
       __threadfence();
@@ -905,29 +969,35 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
 // Depth rows from the level snapshots l in [l0, l1] (l1 capped at the group's last
 // committed level and at 127): depth[j][v] = the first l with bit j of S_l[v] set.
 //
-// A CTA owns a tile of DV consecutive caller-id vertices (columns) x all W rows, staged
-// in a shared [W][DV] byte tile prefilled with -1 (isolated vertices own no snapshot
-// word).  The tile's vertices of degree > 0 are one contiguous range [c0, c0 + k) of
-// compacted ids, so each level's words for the tile are one contiguous run: thread 0
-// fetches them with 1-D TMA bulk copies (cp.async.bulk, DLB levels per stage, DNS stages
-// completing on mbarriers), DNS - 1 jobs ahead of the consumers, across tile boundaries.
-// Consumers are dealt densely over the k vertices (no lane idles on an isolated column):
-// thread t owns vertex slots t%64 and t%64 + 64 for the W/2 instances of half t/64,
-// and accumulates (l + 1) into the byte of every row whose bit first appears at level l
-// (SIMD within a register: bytes never carry, each receives at most one value <= 128).
-// An isolated source gets 0 in its own row.  The tile is written row by row with 16-byte
-// stores (full 128-byte lines).  first != 0 writes every byte; otherwise only the bytes
-// found in [l0, l1] change (a ring-slot flush before reuse).
-constexpr int DV = 128;         // columns per tile
-constexpr int DTHREADS = 128;
+// A CTA owns a tile of DV = 128 consecutive caller-id vertices (columns) x all W rows,
+// staged in a shared [W][128] byte tile (128-byte swizzled, double-buffered) prefilled
+// with -1 (isolated vertices own no snapshot word).  The tile's vertices of degree > 0 are
+// one contiguous range [c0, c0 + k) of compacted ids, so each level's words for the tile
+// are one contiguous run: a producer warp fetches them with 1-D TMA bulk copies
+// (cp.async.bulk, DLB levels per stage, DNS stages on mbarriers), DNS - 1 jobs ahead of
+// the consumers, across tile boundaries.  Consumers are dealt densely over the k
+// vertices (no lane idles on an isolated column): thread t owns vertex slots t%64 and
+// t%64 + 64 for the W/2 instances of half t/64, and accumulates (l + 1) into the byte of
+// every row whose bit first appears at level l (SIMD within a register: bytes never
+// carry, each receives at most one value <= 128).  An isolated source gets 0 in its own
+// row.  The finished tile leaves with one 2-D TMA tensor store (cp.async.bulk.tensor,
+// full 128-byte rows) while the CTA fills the other buffer.  first != 0 writes every
+// byte; otherwise (a ring-slot flush before reuse) only the bytes found in [l0, l1]
+// change, with plain byte stores.
+constexpr int DV = 128;         // columns per tile (= the 128-byte swizzle span)
+constexpr int DTHREADS = 128;   // consumer threads (+ one producer warp)
 constexpr int DLB = 4;          // levels per pipeline stage
 constexpr int DNS = 4;          // pipeline stages (DNS - 1 jobs in flight)
 constexpr int DSLOTS = DTHREADS / 2;  // vertex slots per pass (two halves per vertex)
-constexpr int DROWB = DV + 16;  // bytes per tile row (padded, 16-byte aligned)
 
 __device__ __forceinline__ uint32_t spread4(uint32_t nib) {
   // 4-bit nibble -> 0x01 in each byte whose bit is set
   return (nib * 0x00204081u) & 0x01010101u;
+}
+
+// byte offset of (row r, column c) in a 128-byte-swizzled [rows][128] tile
+__device__ __forceinline__ uint32_t sw128(uint32_t r, uint32_t c) {
+  return r * 128u + ((((c >> 4) ^ r) & 7u) << 4) + (c & 15u);
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -938,6 +1008,9 @@ __device__ __forceinline__ void mbar_init(unsigned long long *bar, uint32_t coun
 __device__ __forceinline__ void mbar_arrive_expect_tx(unsigned long long *bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
                : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned long long *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t parity) {
   asm volatile(
@@ -956,6 +1029,19 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+// 2-D TMA tensor store shared -> global of one box at (x, y), as a bulk group.
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, const void *src, int x, int y) {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(map), "r"(x),
+               "r"(y), "r"(smem_u32(src))
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// barrier among the DTHREADS consumer threads only (the producer warp never joins)
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(DTHREADS) : "memory"); }
 
 // m16n8k32 u8 x u8 -> s32 tensor-core MMA (D += A * B), fragments per the PTX ISA.
 __device__ __forceinline__ void mma_u8_m16n8k32(int (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2,
@@ -993,10 +1079,10 @@ __device__ __forceinline__ void flush_macc(int (&dacc)[NT][4], unsigned long lon
 template <typename T>
 struct DepthLayout {
   static constexpr int W = WordBits<T>::value;
-  static constexpr size_t SROW = (size_t)DV * sizeof(T) + 16;  // one level's run (+ alignment slack)
-  static constexpr size_t TILE = (size_t)W * DROWB;
+  static constexpr size_t TILE = (size_t)W * DV;                     // one output buffer
+  static constexpr size_t SROW = (size_t)DV * sizeof(T) + 16;        // one level's run (+ slack)
   static constexpr size_t STAGE = DLB * SROW;
-  static constexpr size_t BYTES = TILE + DNS * STAGE;
+  static constexpr size_t BYTES = 1024 + 2 * TILE + DNS * STAGE;     // + 1024 for alignment
 };
 
 template <typename T>
@@ -1004,11 +1090,13 @@ constexpr size_t depth_smem_bytes() {
   return DepthLayout<T>::BYTES;
 }
 
-__device__ __forceinline__ void mbar_arrive(unsigned long long *bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+// column (within the tile) of the i-th vertex of degree > 0, from the tile's 4 nzbits words
+__device__ __forceinline__ int dense_col(uint4 w, uint32_t p0, uint32_t p1, uint32_t p2, uint32_t i) {
+  if (i < p0) return (int)__fns(w.x, 0, i + 1);
+  if (i < p1) return 32 + (int)__fns(w.y, 0, i - p0 + 1);
+  if (i < p2) return 64 + (int)__fns(w.z, 0, i - p1 + 1);
+  return 96 + (int)__fns(w.w, 0, i - p2 + 1);
 }
-// barrier among the DTHREADS consumer threads only (the producer warp never joins)
-__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(DTHREADS) : "memory"); }
 
 // The same pass accumulates m_s (reading #11): every byte it finds adds deg(v) to row j's
 // sum (each (j, v) is found in exactly one flush) -- a [4 x DV] x [DV x W] u8 product per
@@ -1018,8 +1106,9 @@ __device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;
 // the bulk copies).  Stage st is "full" when its bytes landed (s_full[st], expect_tx) and
 // "empty" when every consumer warp has read it (s_empty[st], one arrive per warp).
 template <typename T>
-__global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a, int l0, int l1, int first,
-                                                                unsigned long long *m_out) {
+__global__ void __launch_bounds__(DTHREADS + 32, 3)
+    depth_kernel(BatchArgs<T> a, int l0, int l1, int first, unsigned long long *m_out,
+                 const __grid_constant__ CUtensorMap out_map, int use_tma) {
   using L = DepthLayout<T>;
   constexpr int W = WordBits<T>::value;
   constexpr int HQ = W / 8;                        // 32-bit byte registers per (vertex, half)
@@ -1027,13 +1116,12 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
   constexpr int NTILES = W / 8;                    // 8-row n-tiles of the MMA
   constexpr int NTW = NTILES >= NWD ? NTILES / NWD : 1;
   constexpr int MMA_WARPS = NTILES / NTW;          // warps taking part in the MMA
-  extern __shared__ __align__(128) unsigned char dsm[];
-  unsigned char *tb = dsm;                          // [W][DROWB]
-  unsigned char *stage_base = dsm + L::TILE;        // [DNS][DLB][SROW]
+  extern __shared__ unsigned char dsm_raw[];
+  unsigned char *dsm = reinterpret_cast<unsigned char *>(((uintptr_t)dsm_raw + 1023) & ~(uintptr_t)1023);
+  unsigned char *tiles = dsm;                          // [2][W][128], 128B-swizzled
+  unsigned char *stage_base = dsm + 2 * L::TILE;       // [DNS][DLB][SROW]
   __shared__ __align__(8) unsigned long long s_full[DNS], s_empty[DNS];
   __shared__ uint32_t s_deg[DV];
-  __shared__ uint16_t s_col[DV];
-  __shared__ uint32_t s_wcnt[NWD];
   __shared__ unsigned long long s_m[W];
   __shared__ uint32_t s_isrc[W];  // caller id of row j's source if it is isolated, else NO_VERTEX
   __shared__ uint32_t s_has_iso;
@@ -1051,7 +1139,6 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
   int8_t *out = a.out + (size_t)g * W * a.nv;
   const size_t nvv = a.nv;
   const size_t ntiles = (nvv + DV - 1) / DV;
-  const size_t ntb = (nvv + 127) / 128;  // entries of tbase - 1
   const size_t my_tiles = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
   const size_t njobs = my_tiles * (size_t)nbat;
   if (t == 0) {
@@ -1066,8 +1153,7 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
   if (warp == NWD) {
     // ---- producer: job jb = (tile jb / nbat of this CTA, batch jb % nbat) -> stage jb % DNS
     if (lane == 0 && njobs) {
-      uint32_t c0n = __ldg(a.tbase + blockIdx.x * (DV / 128));
-      uint32_t c1n = __ldg(a.tbase + min((size_t)blockIdx.x * (DV / 128) + DV / 128, ntb));
+      uint32_t c0n = __ldg(a.tbase + blockIdx.x), c1n = __ldg(a.tbase + blockIdx.x + 1);
       uint32_t c0 = 0, k = 0;
       for (size_t jb = 0; jb < njobs; ++jb) {
         const int st = (int)(jb % DNS);
@@ -1077,8 +1163,8 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
           k = c1n - c0n;
           const size_t nt = blockIdx.x + (jb / nbat + 1) * gridDim.x;
           if (nt < ntiles) {
-            c0n = __ldg(a.tbase + nt * (DV / 128));
-            c1n = __ldg(a.tbase + min(nt * (DV / 128) + DV / 128, ntb));
+            c0n = __ldg(a.tbase + nt);
+            c1n = __ldg(a.tbase + nt + 1);
           }
         }
         if (jb >= (size_t)DNS) mbar_wait(&s_empty[st], (uint32_t)((jb / DNS - 1) & 1));
@@ -1101,7 +1187,6 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
     }
   } else {
     // ---- consumers
-    const uint32_t *tw = reinterpret_cast<const uint32_t *>(tb);
     int dacc[NTW][4];
 #pragma unroll
     for (int nt = 0; nt < NTW; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
@@ -1116,26 +1201,33 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
       s_isrc[j] = x;
     }
     size_t job = 0;
-    for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x) {
+    int buf = 0;
+    // the tile's 4 nzbits words and compacted base, prefetched one tile ahead
+    uint4 nzw_next = blockIdx.x < ntiles ? __ldg(reinterpret_cast<const uint4 *>(a.nzbits) + blockIdx.x) : uint4{};
+    uint32_t c0_next = blockIdx.x < ntiles ? __ldg(a.tbase + blockIdx.x) : 0u;
+    for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x, buf ^= 1) {
       const size_t v0 = tix * DV;
-      const size_t v = v0 + t;
-      // ranks of the non-isolated columns; prefill -1 (the previous tile is written out)
-      const uint32_t word = v < nvv ? __ldg(a.nzbits + (v >> 5)) : 0u;
-      const bool nz = (word >> lane) & 1u;
-      const uint32_t c0t = __ldg(a.tbase + tix * (DV / 128));
-      if (lane == 0) s_wcnt[warp] = __popc(word);
+      unsigned char *tb = tiles + (size_t)buf * L::TILE;
+      const uint32_t *tw = reinterpret_cast<const uint32_t *>(tb);
+      const uint4 nzw = nzw_next;  // bits beyond nv are 0
+      const uint32_t c0t = c0_next;
+      if (tix + gridDim.x < ntiles) {
+        nzw_next = __ldg(reinterpret_cast<const uint4 *>(a.nzbits) + tix + gridDim.x);
+        c0_next = __ldg(a.tbase + tix + gridDim.x);
+      }
+      const uint32_t p0 = __popc(nzw.x), p1 = p0 + __popc(nzw.y), p2 = p1 + __popc(nzw.z);
+      const uint32_t kcount = p2 + __popc(nzw.w);
+      uint32_t dgr[2];  // degrees of my two slots, in flight during the level batches
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const uint32_t i = slot + DSLOTS * r;
+        dgr[r] = (i < kcount && half == 0) ? __ldg(a.deg + c0t + i) : 0u;
+      }
+      if (t == 0 && use_tma) bulk_wait_read1();  // this buffer's previous store has read it out
+      consumers_sync();                          // ... and the previous tile's readers are done
       s_deg[t] = 0;
       for (int k4 = t; k4 < (int)(L::TILE / 16); k4 += DTHREADS)
         reinterpret_cast<int4 *>(tb)[k4] = make_int4(-1, -1, -1, -1);
-      consumers_sync();
-      uint32_t before = 0, kcount = 0;
-#pragma unroll
-      for (int w = 0; w < NWD; ++w) {
-        const uint32_t x = s_wcnt[w];
-        before += w < warp ? x : 0u;
-        kcount += x;
-      }
-      if (nz) s_col[before + __popc(word & ((1u << lane) - 1u))] = (uint16_t)t;
       uint32_t acc[2][HQ];
 #pragma unroll
       for (int r = 0; r < 2; ++r)
@@ -1167,19 +1259,28 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
         __syncwarp();
         if (lane == 0) mbar_arrive(&s_empty[st]);  // this warp is done with stage st
       }
+      consumers_sync();  // prefill done everywhere before the columns land
       // the tile's columns
 #pragma unroll
       for (int r = 0; r < 2; ++r) {
         const uint32_t i = slot + DSLOTS * r;
         if (i < kcount) {
-          const int col = s_col[i];
-          if (half == 0) s_deg[col] = __ldg(a.deg + c0t + i);
+          const uint32_t col = (uint32_t)dense_col(nzw, p0, p1, p2, i);
+          if (half == 0) s_deg[col] = dgr[r];
+          // swizzled column offset for each row phase (row & 7), so every store below is
+          // base + row * 128 + cs[row & 7] with a compile-time row
+          uint32_t cs[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) cs[k] = ((((col >> 4) ^ (uint32_t)k) & 7u) << 4) + (col & 15u);
+          unsigned char *hb = tb + half * (W / 2) * 128;
 #pragma unroll
           for (int q = 0; q < HQ; ++q) {
             const uint32_t x = __vsub4(acc[r][q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
 #pragma unroll
-            for (int bb = 0; bb < 4; ++bb)
-              tb[(half * (W / 2) + q * 4 + bb) * DROWB + col] = (unsigned char)(x >> (8 * bb));
+            for (int bb = 0; bb < 4; ++bb) {
+              const int row = q * 4 + bb;  // (half * W/2 is a multiple of 8: same phase)
+              hb[row * 128 + cs[row & 7]] = (unsigned char)(x >> (8 * bb));
+            }
           }
         }
       }
@@ -1187,9 +1288,17 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
       if (s_has_iso) {  // isolated sources: depth 0 in their own row (degree 0: no m_s)
         for (int j = t; j < rows; j += DTHREADS) {
           const uint32_t s = s_isrc[j];
-          if (s != NO_VERTEX && s >= v0 && s < v0 + DV) tb[j * DROWB + (s - v0)] = 0;
+          if (s != NO_VERTEX && s >= v0 && s < v0 + DV) tb[sw128(j, s - v0)] = 0;
         }
         consumers_sync();
+      }
+      if (use_tma) {
+        if (t == 0) tma_store_2d(&out_map, tb, (int)v0, g * W);
+      } else if (v0 + t < nvv) {
+        for (int j = 0; j < rows; ++j) {
+          const int8_t d = (int8_t)tb[sw128(j, t)];
+          if (first || d != -1) out[(size_t)j * nvv + v0 + t] = d;
+        }
       }
       // m_s on the tensor cores: D[b][j] += sum_v deg_b(v) * reached(j, v), deg_b = byte b
       // of deg(v) (A: 16 x 32 u8, rows 0..3 = byte planes), reached from the tile (B: 32 x
@@ -1206,8 +1315,10 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
 #pragma unroll
           for (int nt = 0; nt < NTW; ++nt) {
             const int j = (warp * NTW + nt) * 8 + gq;
-            const uint32_t b0 = __vcmpne4(tw[j * (DROWB / 4) + ks * 8 + tq4], 0xffffffffu) & 0x01010101u;
-            const uint32_t b1 = __vcmpne4(tw[j * (DROWB / 4) + ks * 8 + 4 + tq4], 0xffffffffu) & 0x01010101u;
+            const uint32_t w0 = j * 32 + ((((uint32_t)(2 * ks) ^ (uint32_t)j) & 7u) << 2) + tq4;
+            const uint32_t w1 = j * 32 + ((((uint32_t)(2 * ks + 1) ^ (uint32_t)j) & 7u) << 2) + tq4;
+            const uint32_t b0 = __vcmpne4(tw[w0], 0xffffffffu) & 0x01010101u;
+            const uint32_t b1 = __vcmpne4(tw[w1], 0xffffffffu) & 0x01010101u;
             mma_u8_m16n8k32(dacc[nt], a0, 0u, a2, 0u, b0, b1);
           }
         }
@@ -1216,22 +1327,9 @@ __global__ void __launch_bounds__(DTHREADS + 32, 3) depth_kernel(BatchArgs<T> a,
           tiles_acc = 0;
         }
       }
-      const bool vec = first && ((nvv & 15) == 0) && (((uintptr_t)out & 15) == 0) && (v0 + DV <= nvv);
-      if (vec) {
-        // DV/16 threads x 16 bytes per row segment; DTHREADS/(DV/16) rows per pass
-        const int sub = t % (DV / 16), r0 = t / (DV / 16);
-        for (int j = r0; j < rows; j += DTHREADS / (DV / 16))
-          *reinterpret_cast<int4 *>(out + (size_t)j * nvv + v0 + sub * 16) =
-              *reinterpret_cast<const int4 *>(tb + j * DROWB + sub * 16);
-      } else if (v < nvv) {
-        for (int j = 0; j < rows; ++j) {
-          const int8_t d = (int8_t)tb[j * DROWB + t];
-          if (first || d != -1) out[(size_t)j * nvv + v] = d;
-        }
-      }
-      consumers_sync();  // tile and s_deg / s_col reused by the next tile
     }
     if (warp < MMA_WARPS) flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
+    if (t == 0 && use_tma) bulk_wait_all();
   }
   __syncthreads();
   for (int j = t; j < rows; j += DTHREADS)

@@ -229,10 +229,16 @@ def main():
 
     # ---- roofline of the dominant kernel (algorithmic bytes / CUDA-event time) -------
     peak, peak_kind = peak_hbm()
+    # level_kernel = commit of level l-1 + expand of level l (one cooperative launch per
+    # level); its two phases are also split by the kernel's own globaltimer stamps
     kern = {
-        "expand": (sum(s.expand_bytes for s in sts), sum(s.expand_ms for s in sts), sum(s.expand_launches for s in sts)),
-        "commit": (sum(s.commit_bytes for s in sts), sum(s.commit_ms for s in sts), sum(s.commit_launches for s in sts)),
+        "level": (sum(s.expand_bytes + s.commit_bytes for s in sts), sum(s.level_ms for s in sts),
+                  sum(s.level_launches for s in sts)),
         "depth": (sum(s.depth_bytes for s in sts), sum(s.depth_ms for s in sts), sum(s.depth_launches for s in sts)),
+    }
+    phases = {
+        "level.expand": (sum(s.expand_bytes for s in sts), sum(s.expand_ms for s in sts)),
+        "level.commit": (sum(s.commit_bytes for s in sts), sum(s.commit_ms for s in sts)),
     }
     dom = max(kern, key=lambda k: kern[k][1])
     b, ms, nl = kern[dom]
@@ -243,7 +249,9 @@ def main():
                 "traffic": traffic, "algorithmic_bytes_per_launch": (b / nl if nl else None),
                 "share_of_step": round(ms / local_ms, 4) if local_ms else None,
                 "all_kernels": {k: {"GB/s": round(v[0] / (v[1] * 1e-3) / 1e9, 1) if v[1] else None,
-                                    "ms": round(v[1], 3), "launches": v[2]} for k, v in kern.items()}}
+                                    "ms": round(v[1], 3), "launches": v[2]} for k, v in kern.items()},
+                "phases": {k: {"GB/s": round(v[0] / (v[1] * 1e-3) / 1e9, 1) if v[1] else None,
+                               "ms": round(v[1], 3)} for k, v in phases.items()}}
 
     # ---- end to end through the public API with HOST buffers -------------------------
     e2e = None

@@ -179,9 +179,12 @@ typedef struct {
   uint32_t n_groups, max_levels;
   uint32_t levels_td, levels_bu;  /* group-levels run in each direction */
   uint64_t n_launches;            /* kernels this call launched (traversal + finalize) */
-  /* per-kernel device time and algorithmic bytes (bytes always; ms only if opts.timing) */
-  double expand_ms, commit_ms, init_ms, depth_ms;
-  uint64_t expand_launches, commit_launches, init_launches, depth_launches;
+  /* per-kernel device time and algorithmic bytes.  One level_kernel launch per level runs
+     the commit of level l-1 and the expand of level l (bytes: commit_bytes + expand_bytes);
+     level_ms / init_ms / depth_ms are CUDA-event times (opts.timing only); expand_ms and
+     commit_ms split level time by the kernel's own globaltimer stamps (always). */
+  double level_ms, expand_ms, commit_ms, init_ms, depth_ms;
+  uint64_t level_launches, init_launches, depth_launches;
   uint64_t expand_bytes, commit_bytes, init_bytes, depth_bytes;
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */

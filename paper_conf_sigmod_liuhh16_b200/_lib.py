@@ -55,10 +55,9 @@ class Stats(C.Structure):
                 ("sd_jfq_bu", C.c_uint64),
                 ("n_groups", C.c_uint32), ("max_levels", C.c_uint32), ("levels_td", C.c_uint32),
                 ("levels_bu", C.c_uint32), ("n_launches", C.c_uint64),
-                ("expand_ms", C.c_double), ("commit_ms", C.c_double), ("init_ms", C.c_double),
-                ("depth_ms", C.c_double),
-                ("expand_launches", C.c_uint64), ("commit_launches", C.c_uint64),
-                ("init_launches", C.c_uint64), ("depth_launches", C.c_uint64),
+                ("level_ms", C.c_double), ("expand_ms", C.c_double), ("commit_ms", C.c_double),
+                ("init_ms", C.c_double), ("depth_ms", C.c_double),
+                ("level_launches", C.c_uint64), ("init_launches", C.c_uint64), ("depth_launches", C.c_uint64),
                 ("expand_bytes", C.c_uint64), ("commit_bytes", C.c_uint64), ("init_bytes", C.c_uint64),
                 ("depth_bytes", C.c_uint64),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),

@@ -5,7 +5,8 @@
 //   groups = consecutive chunks of group_bits sources; G groups run per launch batch
 //   (all of a batch's groups share each level launch; each keeps its own direction).
 //   per batch: init_state + init_sources, then per level l = 1, 2, ...:
-//     expand_kernel(l), commit_kernel(l); every LEVELS_PER_CHECK levels the batch's
+//     level_kernel(l) -- one cooperative launch: commit of level l-1, grid barrier,
+//     expand of level l (kernels.cuh); every LEVELS_PER_CHECK levels the batch's
 //     done-counter is copied to pinned host memory, with one chunk of look-ahead so the
 //     device never waits for the host; kernels of a finished batch exit immediately.
 //   then m_s (+ digest) finalize outside the timed window; D2H of rows if the caller's
@@ -184,7 +185,7 @@ struct ibfs_graph {
   std::vector<uint64_t> h_off;      // host copy of d_off (tiling, planner)
   std::vector<uint32_t> h_tbase, h_nzbits;
   int num_sms = 148;
-  int expand_blocks_per_sm = 1;
+  int level_blocks_per_sm[3] = {1, 1, 1};  // co-resident level_kernel CTAs per SM (W = 32, 64, 128)
 };
 
 namespace {
@@ -381,11 +382,11 @@ void finish_graph(ibfs_graph *g) {
   build_decomposition(g);
   int dev = g->device;
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev));
-  CK(cudaFuncSetAttribute(expand_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  CK(cudaFuncSetAttribute(level_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)sizeof(TileQueue<uint32_t>)));
-  CK(cudaFuncSetAttribute(expand_kernel<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  CK(cudaFuncSetAttribute(level_kernel<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)sizeof(TileQueue<unsigned long long>)));
-  CK(cudaFuncSetAttribute(expand_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  CK(cudaFuncSetAttribute(level_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)sizeof(TileQueue<u128>)));
   CK(cudaFuncSetAttribute(depth_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)depth_smem_bytes<uint32_t>()));
@@ -394,8 +395,13 @@ void finish_graph(ibfs_graph *g) {
   CK(cudaFuncSetAttribute(depth_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)depth_smem_bytes<u128>()));
   int occ = 1;
-  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, expand_kernel<u128>, BLOCK, sizeof(TileQueue<u128>)));
-  g->expand_blocks_per_sm = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_kernel<uint32_t>, BLOCK, sizeof(TileQueue<uint32_t>)));
+  g->level_blocks_per_sm[0] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_kernel<unsigned long long>, BLOCK,
+                                                   sizeof(TileQueue<unsigned long long>)));
+  g->level_blocks_per_sm[1] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_kernel<u128>, BLOCK, sizeof(TileQueue<u128>)));
+  g->level_blocks_per_sm[2] = std::max(1, occ);
   set_pool_threshold(dev);
 }
 
@@ -904,11 +910,13 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
   LevelStat *lstat = sc.get<LevelStat>((size_t)G * MAXL);
   uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
-  uint32_t *flags = sc.get<uint32_t>(2);  // batch_done, range_err
+  uint32_t *flags = sc.get<uint32_t>(4);  // batch_done, range_err, grid barrier (count, generation)
+  unsigned long long *tstamp = sc.get<unsigned long long>((size_t)MAXL * 3);
+  std::vector<unsigned long long> h_ts((size_t)MAXL * 3);
   unsigned long long *d_m = sc.get<unsigned long long>((size_t)G * W);
   unsigned long long *d_dig = sc.get<unsigned long long>((size_t)G * W);
   int8_t *staging = out_dev ? nullptr : sc.get<int8_t>((size_t)G * rows_bytes_per_group);
-  CK(cudaMemsetAsync(flags, 0, 8, stream));
+  CK(cudaMemsetAsync(flags, 0, 16, stream));
 
   DevCache &dc = t_cache.get(g->device);
   if (!dc.pinned) CK(cudaMallocHost(&dc.pinned, 4096));
@@ -934,6 +942,8 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.work_ctr = work_ctr;
   a.batch_done = flags;
   a.range_err = flags + 1;
+  a.gbar = flags + 2;
+  a.tstamp = tstamp;
   a.n_total = n;
   a.chunks = g->d_chunks;
   a.n_chunks = g->n_chunks;
@@ -956,10 +966,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   if (o.direction == IBFS_DIR_BU_FROM) first_dir = o.bu_from <= 1 ? 1 : 0;
   if (o.direction == IBFS_DIR_SCHEDULE && a.pol.sched_len > 0) first_dir = a.pol.sched[0];
 
-  const int expand_grid = g->num_sms * g->expand_blocks_per_sm;
+  const int level_grid = g->num_sms * g->level_blocks_per_sm[W == 32 ? 0 : (W == 64 ? 1 : 2)];
   EventTimer timer(dc, true), chk(dc, false);
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, kexp, kcom, kinit, kdep, kfin;
-  std::vector<int> klev;  // level of each timed expand/commit pair
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin;
   ibfs_stats st{};
   uint64_t launches = 0;
   bool range_error = false;
@@ -990,8 +999,6 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
       st.init_bytes += (uint64_t)Gb * (3 * (uint64_t)nva * B);
       if (o.timing) { CK(cudaEventRecord(i1, stream)); kinit.push_back({i0, i1}); }
     }
-    const uint32_t commit_bx = (uint32_t)std::max<uint64_t>(
-        1, std::min<uint64_t>(((uint64_t)nva + BLOCK * 4 - 1) / (BLOCK * 4), (uint64_t)g->num_sms * 8 / Gb));
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
     // the rows of this batch as a [rows_in_batch][nv] byte tensor for the depth kernel's TMA
@@ -1020,22 +1027,21 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     while (level <= MAXL - 1) {
       const int lend = std::min(level + LEVELS_PER_CHECK, MAXL);
       for (int l = level; l < lend; ++l) {
-        // commit l zeroes slot (l+1) % R, which held level l+1-R: flush it first
-        if (l + 1 - (int)R > flushed) flush(l - 1);
-        cudaEvent_t e0 = nullptr, e1 = nullptr, e2 = nullptr;
-        if (o.timing) { e0 = timer.next(); e1 = timer.next(); e2 = timer.next(); CK(cudaEventRecord(e0, stream)); }
-        expand_kernel<T><<<expand_grid, BLOCK, sizeof(TileQueue<T>), stream>>>(a, l);
-        if (o.timing) CK(cudaEventRecord(e1, stream));
-        commit_kernel<T><<<dim3(commit_bx, Gb), BLOCK, 0, stream>>>(a, l);
+        // level l's commit (of level l-1) zeroes slot l % R, which held level l-R: flush it
+        // first (levels <= l-2 are committed by then)
+        if (l - (int)R > flushed) flush(l - 2);
+        cudaEvent_t e0 = nullptr, e1 = nullptr;
+        if (o.timing) { e0 = timer.next(); e1 = timer.next(); CK(cudaEventRecord(e0, stream)); }
+        int lv = l;
+        void *kargs[] = {(void *)&a, (void *)&lv};
+        CK(cudaLaunchCooperativeKernel((const void *)level_kernel<T>, dim3(level_grid), dim3(BLOCK), kargs,
+                                       sizeof(TileQueue<T>), stream));
         if (o.timing) {
-          CK(cudaEventRecord(e2, stream));
-          kexp.push_back({e0, e1});
-          kcom.push_back({e1, e2});
-          klev.push_back(l);
+          CK(cudaEventRecord(e1, stream));
+          klev.push_back({e0, e1});
         }
-        launches += 2;
-        st.expand_launches++;
-        st.commit_launches++;
+        launches += 1;
+        st.level_launches++;
       }
       CK(cudaGetLastError());
       if (chunk >= 256) fail(IBFS_E_CUDA, "level loop overflow");
@@ -1068,6 +1074,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     CK(cudaEventRecord(f1, stream));
     kfin.push_back({f0, f1});
     CK(cudaMemcpyAsync(h_lstat.data(), lstat, (size_t)Gb * MAXL * sizeof(LevelStat), cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(h_ts.data(), tstamp, (size_t)MAXL * 3 * 8, cudaMemcpyDeviceToHost, stream));
     CK(cudaMemcpyAsync(h_m.data(), d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
     if (stats && stats->per_source_digest)
       CK(cudaMemcpyAsync(h_dig.data(), d_dig, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
@@ -1112,19 +1119,24 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         st.commit_bytes += cb;
       }
     }
+    // phase times of each level kernel from its in-kernel globaltimer stamps: [first CTA
+    // start, grid barrier, last CTA end]; the commit part belongs to level l-1
+    for (int l = 1; l < MAXL; ++l) {
+      const unsigned long long t0 = h_ts[(size_t)l * 3], t1 = h_ts[(size_t)l * 3 + 1], t2 = h_ts[(size_t)l * 3 + 2];
+      if (t0 == ~0ull || t1 < t0 || t2 < t1) continue;
+      const double cms = (t1 - t0) * 1e-6, ems = (t2 - t1) * 1e-6;
+      st.expand_ms += ems;
+      per_level[l - 1].expand_ms += ems;
+      if (l > 1) {
+        st.commit_ms += cms;
+        per_level[l - 2].commit_ms += cms;
+      }
+    }
   }
   if (range_error) fail(IBFS_E_RANGE, "a depth exceeds 127 (int8 output)");
   // times
   for (auto &p : win) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.traverse_ms += ms; }
-  for (size_t i = 0; i < kexp.size(); ++i) {
-    float me = 0, mc = 0;
-    CK(cudaEventElapsedTime(&me, kexp[i].first, kexp[i].second));
-    CK(cudaEventElapsedTime(&mc, kcom[i].first, kcom[i].second));
-    st.expand_ms += me;
-    st.commit_ms += mc;
-    per_level[klev[i] - 1].expand_ms += me;
-    per_level[klev[i] - 1].commit_ms += mc;
-  }
+  for (auto &p : klev) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.level_ms += ms; }
   for (auto &p : kinit) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.init_ms += ms; }
   for (auto &p : kfin) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.finalize_ms += ms; }
   for (auto &p : kdep) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.depth_ms += ms; }

@@ -124,6 +124,8 @@ struct BatchArgs {
   const uint32_t *hub_chunk0;  // [n_hubs + 1] first chunk of each hub (chunks are in hub order)
   uint32_t n_hubs;
   uint32_t *chq;               // [gcap][2][n_chunks] hub-chunk queues (TD, BU)
+  uint32_t *gbar;              // [2] grid barrier (count, generation)
+  unsigned long long *tstamp;  // [MAXL][3] globaltimer: first CTA start, barrier, last CTA end
   uint32_t n_iso;       // vertices of degree 0 (nv - nva)
   Policy pol;
 };
@@ -279,7 +281,12 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     if (done) atomicAdd(a.batch_done, 1u);
   }
   if (g == 0)
-    for (int l = threadIdx.x; l < MAXL; l += blockDim.x) a.work_ctr[l] = 0;
+    for (int l = threadIdx.x; l < MAXL; l += blockDim.x) {
+      a.work_ctr[l] = 0;
+      a.tstamp[(size_t)l * 3] = ~0ull;  // level kernels atomicMin their start here
+      a.tstamp[(size_t)l * 3 + 1] = 0;
+      a.tstamp[(size_t)l * 3 + 2] = 0;
+    }
 }
 
 // Zero the group's visited words and the snapshot slots of levels 0 and 1 (a2); when
@@ -684,17 +691,12 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
   flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tg) : 0u, first ? 1u : 0u, insp, writes);
 }
 
-// One launch per level for all groups of a batch.  Work items, pulled by CTAs from a
-// per-level counter: all hub chunks first, then heavy-queue items, then light-queue
-// items, each carrying its group (whose direction the previous commit decided).
+// Expand phase of level `level` for all groups of a batch.  Work items, pulled by CTAs
+// from a per-level counter: frontier hub chunks first, then heavy-queue items, then
+// light-queue items, each carrying its group (whose direction the commit decided).
 template <typename T>
-__global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) expand_kernel(BatchArgs<T> a, int level) {
-  __shared__ ExpandSmem sm;
-  __shared__ T s_red[NWARP];
-  extern __shared__ __align__(16) unsigned char dyn_smem[];
-  TileQueue<T> &tq = *reinterpret_cast<TileQueue<T> *>(dyn_smem);
+__device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T *s_red, TileQueue<T> &tq) {
   const int tid = threadIdx.x;
-  if (*(volatile uint32_t *)a.batch_done >= (uint32_t)a.G) return;
   for (int i = tid; i < a.G * 5; i += BLOCK) sm.acc[i / 5][i % 5] = 0ull;
   const int par = (level - 1) & 1;  // queues were produced by commit l-1 (or init)
   if (tid == 0) {
@@ -795,144 +797,162 @@ __device__ __forceinline__ bool decide_bu(const Policy &p, uint32_t next_level, 
 // with an unvisited bit of an instance active before this level (a superset of the
 // active set after it: the expand masks with the final one, Lemma C3.5).
 template <typename T>
-__global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level) {
-  __shared__ unsigned long long s_red[NWARP][3];
-  __shared__ T s_or[NWARP];
-  __shared__ uint32_t s_last;
-  __shared__ uint32_t s_wcnt[NWARP][4];
-  __shared__ uint32_t s_qbase[4];
-  const int g = blockIdx.y;
+struct CommitSmem {
+  unsigned long long red[NWARP][3];
+  T orr[NWARP];
+  uint32_t last;
+  uint32_t wcnt[NWARP][4];
+  uint32_t qbase[4];
+};
+
+// Commit of level lc for one tile of group g: the CVT * BLOCK vertices from `base`.
+// visited |= S_lc, zero slot lc + 1, build both JFQs of level lc + 1 -- top-down: vertices
+// with new bits; bottom-up: vertices with an unvisited bit of an instance active before
+// this level (a superset of the active set after it: the expand masks with the final
+// one, Lemma C3.5); hubs go to the hub-chunk queues.  The four vertex-queue classes are
+// appended with one atomic per class per tile (block-wide ballot prefix).  Counters
+// (n_f, m_f, new pairs, OR of new bits) accumulate in the caller's registers.
+constexpr int CVT = 4;
+constexpr int CTILE = CVT * BLOCK;  // vertices per commit tile
+
+template <typename T>
+__device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, size_t base,
+                                            unsigned long long &nf, unsigned long long &mf,
+                                            unsigned long long &newp, T &nacc) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   GroupCtrl<T> *c = a.ctrl + g;
-  if (*(volatile uint32_t *)&c->done) return;
   const T active = c->active;
-  const T *N = next_buf(a, g, level);
-  T *Z = snap(a, g, level + 1);  // target of the next level's expand
+  T *N = snap(a, g, lc);
+  T *Z = snap(a, g, lc + 1);  // target of the next level's expand
   T *vis = a.visited + (size_t)g * a.gstride;
-  uint32_t *qlen = c->qlen[level & 1];
+  uint32_t *qlen = c->qlen[lc & 1];
   const size_t nv = a.nva;
-  unsigned long long nf = 0, mf = 0, newp = 0;
-  T nacc = wzero_value<T>();
-  const size_t stride = (size_t)gridDim.x * BLOCK;
-  // CVT vertices per thread per block iteration; the four queue classes are appended
-  // with one atomic per class per block iteration (block-wide ballot prefix).
-  constexpr int CVT = 4;
-  for (size_t base = (size_t)blockIdx.x * BLOCK * CVT; base < nv; base += stride * CVT) {
-    T n[CVT], vv[CVT];
-    uint32_t dg[CVT];
+  T n[CVT], vv[CVT];
+  uint32_t dg[CVT];
 #pragma unroll
-    for (int k = 0; k < CVT; ++k) {
-      const size_t v = base + (size_t)k * BLOCK + tid;
-      n[k] = wzero_value<T>();
-      vv[k] = wzero_value<T>();
-      dg[k] = 0;
-      if (v < nv) {
-        n[k] = ld(N + v);
-        vv[k] = ld(vis + v);
-        dg[k] = __ldg(a.deg + v);
-      }
+  for (int k = 0; k < CVT; ++k) {
+    const size_t v = base + (size_t)k * BLOCK + tid;
+    n[k] = wzero_value<T>();
+    vv[k] = wzero_value<T>();
+    dg[k] = 0;
+    if (v < nv) {
+      n[k] = ld(N + v);
+      vv[k] = ld(vis + v);
+      dg[k] = __ldg(a.deg + v);
     }
-    uint32_t bal[CVT][4];
-    uint32_t wc[4] = {0, 0, 0, 0};
+  }
+  uint32_t bal[CVT][4];
+  uint32_t wc[4] = {0, 0, 0, 0};
 #pragma unroll
-    for (int k = 0; k < CVT; ++k) {
-      const size_t v = base + (size_t)k * BLOCK + tid;
-      const bool in = v < nv;
-      if (in) st(Z + v, wzero_value<T>());
-      {  // an unfiltered top-down level may have ORed already-visited bits: mask them
-        const T m = wandn(n[k], vv[k]);
-        if (in && !weq(m, n[k])) st(const_cast<T *>(N) + v, m);
-        n[k] = m;
-      }
-      const bool nz = !wzero(n[k]);
-      if (nz) st(vis + v, wor(vv[k], n[k]));
-      const T tp = in ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
-      const bool un = !wzero(tp);
-      const uint32_t d = dg[k];
-      if (nz) {
-        nf++;
-        mf += d;
-        newp += wpopc(n[k]);
-        nacc = wor(nacc, n[k]);
-      }
-      const bool qd = d > 0 && d <= (uint32_t)HUB_T;
-      const bool light = d <= (uint32_t)LIGHT_DEG;
-      bal[k][Q_TDL] = __ballot_sync(FULL, nz && qd && light);
-      bal[k][Q_TDH] = __ballot_sync(FULL, nz && qd && !light);
-      bal[k][Q_BUL] = __ballot_sync(FULL, un && qd && light);
-      bal[k][Q_BUH] = __ballot_sync(FULL, un && qd && !light);
-      // hubs: their chunks, never the vertex queues
+  for (int k = 0; k < CVT; ++k) {
+    const size_t v = base + (size_t)k * BLOCK + tid;
+    const bool in = v < nv;
+    if (in) st(Z + v, wzero_value<T>());
+    {  // an unfiltered top-down level may have ORed already-visited bits: mask them
+      const T m = wandn(n[k], vv[k]);
+      if (in && !weq(m, n[k])) st(N + v, m);
+      n[k] = m;
+    }
+    const bool nz = !wzero(n[k]);
+    if (nz) st(vis + v, wor(vv[k], n[k]));
+    const T tp = in ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
+    const bool un = !wzero(tp);
+    const uint32_t d = dg[k];
+    if (nz) {
+      nf++;
+      mf += d;
+      newp += wpopc(n[k]);
+      nacc = wor(nacc, n[k]);
+    }
+    const bool qd = d > 0 && d <= (uint32_t)HUB_T;
+    const bool light = d <= (uint32_t)LIGHT_DEG;
+    bal[k][Q_TDL] = __ballot_sync(FULL, nz && qd && light);
+    bal[k][Q_TDH] = __ballot_sync(FULL, nz && qd && !light);
+    bal[k][Q_BUL] = __ballot_sync(FULL, un && qd && light);
+    bal[k][Q_BUH] = __ballot_sync(FULL, un && qd && !light);
+    // hubs: their chunks, never the vertex queues (rare: one vote in the common case)
+    if (__any_sync(FULL, in && d > (uint32_t)HUB_T)) {
       push_hub_chunks(a, g, qlen, Q_TDC, in && nz && d > (uint32_t)HUB_T, (uint32_t)v);
       push_hub_chunks(a, g, qlen, Q_BUC, in && un && d > (uint32_t)HUB_T, (uint32_t)v);
-#pragma unroll
-      for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
     }
-    if (lane == 0)
-      for (int cls = 0; cls < 4; ++cls) s_wcnt[warp][cls] = wc[cls];
-    __syncthreads();
-    if (tid < 4) {
-      uint32_t tot = 0;
-      for (int w = 0; w < NWARP; ++w) {
-        const uint32_t x = s_wcnt[w][tid];
-        s_wcnt[w][tid] = tot;  // exclusive warp offsets
-        tot += x;
-      }
-      s_qbase[tid] = tot ? atomicAdd(qlen + tid, tot) : 0u;
-    }
-    __syncthreads();
 #pragma unroll
-    for (int cls = 0; cls < 4; ++cls) {
-      uint32_t off = s_qbase[cls] + s_wcnt[warp][cls];
-      uint32_t *q = queue_of(a, g, cls);
-#pragma unroll
-      for (int k = 0; k < CVT; ++k) {
-        const uint32_t b = bal[k][cls];
-        if ((b >> lane) & 1u) {
-          const uint32_t i = off + __popc(b & lanemask_lt());
-          const uint32_t v = (uint32_t)(base + (size_t)k * BLOCK + tid);
-          if (cls & 1) q[nv - 1 - i] = v; else q[i] = v;
-        }
-        off += __popc(b);
-      }
-    }
-    __syncthreads();  // s_wcnt / s_qbase reused next iteration
+    for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
   }
-  if (level >= 128 && !wzero(nacc)) atomicExch(a.range_err, 1u);  // depth > 127
+  if (lane == 0)
+    for (int cls = 0; cls < 4; ++cls) cm.wcnt[warp][cls] = wc[cls];
+  __syncthreads();
+  if (tid < 4) {
+    uint32_t tot = 0;
+    for (int w = 0; w < NWARP; ++w) {
+      const uint32_t x = cm.wcnt[w][tid];
+      cm.wcnt[w][tid] = tot;  // exclusive warp offsets
+      tot += x;
+    }
+    cm.qbase[tid] = tot ? atomicAdd(qlen + tid, tot) : 0u;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int cls = 0; cls < 4; ++cls) {
+    uint32_t off = cm.qbase[cls] + cm.wcnt[warp][cls];
+    uint32_t *q = queue_of(a, g, cls);
+#pragma unroll
+    for (int k = 0; k < CVT; ++k) {
+      const uint32_t b = bal[k][cls];
+      if ((b >> lane) & 1u) {
+        const uint32_t i = off + __popc(b & lanemask_lt());
+        const uint32_t v = (uint32_t)(base + (size_t)k * BLOCK + tid);
+        if (cls & 1) q[nv - 1 - i] = v; else q[i] = v;
+      }
+      off += __popc(b);
+    }
+  }
+  __syncthreads();  // wcnt / qbase reused by the next tile
+}
+
+// Add one CTA's counters for group g (ntiles tiles) to the group, and if they complete the
+// group's tiles, decide the next level: direction (reading #7), active mask, done.
+template <typename T>
+__device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, uint32_t ntiles,
+                             uint32_t tiles_per_group, unsigned long long nf, unsigned long long mf,
+                             unsigned long long newp, T nacc) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  GroupCtrl<T> *c = a.ctrl + g;
+  if (lc >= 128 && !wzero(nacc)) atomicExch(a.range_err, 1u);  // depth > 127
   nf = warp_sum64(nf);
   mf = warp_sum64(mf);
   newp = warp_sum64(newp);
   nacc = warp_or(nacc);
   if (lane == 0) {
-    s_red[warp][0] = nf; s_red[warp][1] = mf; s_red[warp][2] = newp;
-    s_or[warp] = nacc;
+    cm.red[warp][0] = nf; cm.red[warp][1] = mf; cm.red[warp][2] = newp;
+    cm.orr[warp] = nacc;
   }
   __syncthreads();
   if (tid == 0) {
     unsigned long long t0 = 0, t1 = 0, t2 = 0;
     T o = wzero_value<T>();
     for (int k = 0; k < NWARP; ++k) {
-      t0 += s_red[k][0]; t1 += s_red[k][1]; t2 += s_red[k][2];
-      o = wor(o, s_or[k]);
+      t0 += cm.red[k][0]; t1 += cm.red[k][1]; t2 += cm.red[k][2];
+      o = wor(o, cm.orr[k]);
     }
     if (t0) atomicAdd(&c->n_f, t0);
     if (t1) atomicAdd(&c->m_f, t1);
     if (t2) atomicAdd(&c->newp, t2);
     if (!wzero(o)) red_or(&c->newacc, o);
     __threadfence();
-    const uint32_t prev = atomicAdd(&c->arrive, 1u);
-    s_last = (prev == gridDim.x - 1) ? 1u : 0u;
+    const uint32_t prev = atomicAdd(&c->arrive, ntiles);
+    cm.last = (prev + ntiles == tiles_per_group) ? 1u : 0u;
   }
   __syncthreads();
-  if (s_last && tid == 0) {
+  if (cm.last && tid == 0) {
     __threadfence();
     const T act = ldv(&c->newacc);
     const unsigned long long n_f = ldv(&c->n_f), m_f = ldv(&c->m_f), np = ldv(&c->newp);
     const uint32_t cur = c->dir;
-    LevelStat *ls = a.lstat + (size_t)g * MAXL + level;
+    LevelStat *ls = a.lstat + (size_t)g * MAXL + lc;
     ls->dir = cur + 1;
     ls->newp = np;
     ls->nf = n_f;
-    const bool bu = decide_bu(a.pol, (uint32_t)level + 1, cur, n_f, m_f);
+    const bool bu = decide_bu(a.pol, (uint32_t)lc + 1, cur, n_f, m_f);
     c->active = act;
     c->newacc = wzero_value<T>();
     c->n_f = c->m_f = c->newp = 0;
@@ -943,17 +963,17 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
     c->vpairs += np;
     c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
-    c->last_level = (uint32_t)level;
-    for (int k = 0; k < NQ; ++k) c->qlen[(level + 1) & 1][k] = 0;  // target of commit l+1
+    c->last_level = (uint32_t)lc;
+    for (int k = 0; k < NQ; ++k) c->qlen[(lc + 1) & 1][k] = 0;  // target of commit lc+1
     if (wzero(act)) {
       c->done = 1;
       __threadfence();
       atomicAdd(a.batch_done, 1u);
-    } else if (level + 1 < MAXL) {
-      // Eq. 1 counters of level l+1 known here: TD -- |JFQ| = vertices with new bits,
+    } else if (lc + 1 < MAXL) {
+      // Eq. 1 counters of level lc+1 known here: TD -- |JFQ| = vertices with new bits,
       // sum_j |FQ_j| = new pairs; BU -- the isolated vertices (never in the queues; every
       // active instance is unvisited there), the expand adds the queued ones and hubs.
-      LevelStat *nx = a.lstat + (size_t)g * MAXL + level + 1;
+      LevelStat *nx = a.lstat + (size_t)g * MAXL + lc + 1;
       if (!bu) {
         nx->jfq = n_f;
         nx->fq = np;
@@ -962,6 +982,94 @@ __global__ void __launch_bounds__(BLOCK) commit_kernel(BatchArgs<T> a, int level
         nx->fq = (unsigned long long)a.n_iso * (unsigned long long)wpopc(act);
       }
     }
+  }
+}
+
+// Grid-wide barrier of a cooperative launch (every CTA resident): sense-reversing, one
+// counter and one generation word per batch.
+__device__ __forceinline__ void grid_barrier(uint32_t *bar) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    volatile uint32_t *gen = bar + 1;
+    const uint32_t my_gen = *gen;
+    __threadfence();
+    const uint32_t nb = gridDim.x * gridDim.y;
+    if (atomicAdd(bar, 1u) == nb - 1) {
+      bar[0] = 0;
+      __threadfence();
+      atomicAdd(bar + 1, 1u);
+    } else {
+      while (*gen == my_gen) __nanosleep(32);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+// ---------------------------------------------------------------------- level ----
+// THE per-level kernel (north_star: "a single kernel per level builds the joint frontier
+// queue and expands it"), one cooperative launch for all groups of a batch:
+//   phase 1 (level > 1): commit of level l-1 over every (group, vertex tile) -- visited
+//            |= S_l-1, zero slot l, build the JFQs of level l (Alg. 2), counters; the CTA
+//            completing a group decides its direction for level l;
+//   grid barrier (the expand must see committed words: Lemma C2, reading #4);
+//   phase 2: expand of level l (Alg. 1) from those queues.
+// Level 1's queues come from the init kernels.  A batch whose groups are all finished
+// (flags final before this launch) exits at once.
+template <typename T>
+__global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArgs<T> a, int level) {
+  __shared__ ExpandSmem sm;
+  __shared__ T s_red[NWARP];
+  __shared__ CommitSmem<T> cm;
+  __shared__ uint32_t s_live;
+  extern __shared__ __align__(16) unsigned char dyn_smem[];
+  TileQueue<T> &tq = *reinterpret_cast<TileQueue<T> *>(dyn_smem);
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    uint32_t live = 0;
+    for (int g = 0; g < a.G; ++g) live += a.ctrl[g].done ? 0u : 1u;
+    s_live = live;
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (live) atomicMin(a.tstamp + (size_t)level * 3, t);
+  }
+  __syncthreads();
+  if (s_live == 0) return;  // uniform: every CTA reads the same final flags
+  if (level > 1) {
+    const int lc = level - 1;
+    const uint32_t tpg = (uint32_t)((a.nva + CTILE - 1) / CTILE);
+    const size_t total = (size_t)a.G * tpg;
+    int cur_g = -1;
+    uint32_t ntiles = 0;
+    unsigned long long nf = 0, mf = 0, newp = 0;
+    T nacc = wzero_value<T>();
+    for (size_t w = blockIdx.x; w < total; w += gridDim.x) {
+      const int g = (int)(w / tpg);
+      if (g != cur_g) {
+        if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc);
+        cur_g = g;
+        ntiles = 0;
+        nf = mf = newp = 0;
+        nacc = wzero_value<T>();
+      }
+      if (a.ctrl[g].done) continue;  // finished before this launch (stable)
+      commit_tile(a, cm, g, lc, (size_t)(w % tpg) * CTILE, nf, mf, newp, nacc);
+      ++ntiles;
+    }
+    if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc);
+    grid_barrier(a.gbar);
+  }
+  if (tid == 0 && blockIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    a.tstamp[(size_t)level * 3 + 1] = t;
+  }
+  expand_phase(a, level, sm, s_red, tq);
+  __syncthreads();
+  if (tid == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    atomicMax(a.tstamp + (size_t)level * 3 + 2, t);
   }
 }
 

@@ -76,12 +76,12 @@ class RunStats:
     levels_td: int
     levels_bu: int
     n_launches: int
+    level_ms: float
     expand_ms: float
     commit_ms: float
     init_ms: float
     depth_ms: float
-    expand_launches: int
-    commit_launches: int
+    level_launches: int
     init_launches: int
     depth_launches: int
     expand_bytes: int

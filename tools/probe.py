@@ -25,7 +25,7 @@ for it in range(iters):
     _, st = g.run(ss, 128, out=out[: len(ss)], timing=True, **kw)
     t1 = time.perf_counter()
     print(f"{name} it{it}: wall {1e3*(t1-t0):.1f} ms traverse {st.traverse_ms:.1f} finalize {st.finalize_ms:.1f} "
-          f"expand {st.expand_ms:.1f} commit {st.commit_ms:.1f} depth {st.depth_ms:.1f} init {st.init_ms:.1f} "
+          f"level {st.level_ms:.1f} (expand {st.expand_ms:.1f} commit {st.commit_ms:.1f}) depth {st.depth_ms:.1f} init {st.init_ms:.1f} "
           f"levels {st.max_levels} td {st.levels_td} bu {st.levels_bu} gteps {st.gteps:.0f} launches {st.n_launches}")
     for i, L in enumerate(st.per_level):
         print("   L%d td%d bu%d jfq_td %d jfq_bu %d insp %d new %d  exp %.2f ms com %.2f ms" % (i + 1, L["td_groups"], L["bu_groups"], L["jfq_td"], L["jfq_bu"], L["inspected"], L["new_pairs"], L["expand_ms"], L["commit_ms"]))

@@ -32,7 +32,7 @@ sys.path.insert(0, ROOT)
 import ibfs_gen  # noqa: E402  (seeded input generator shared with the oracle)
 
 METRIC = "aggregate GTEPS (summed over i instances)"
-DEFAULT_GROUPS = {"c1": 1, "c2": 1, "c3": 8, "c4": 256, "c5": 2}
+DEFAULT_GROUPS = {"c1": 1, "c2": 1, "c3": 8, "c4": 256, "c5": 4}
 PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM = 6650.0  # GB/s, B200_PROFILING.md fallback
 
@@ -40,7 +40,7 @@ FALLBACK_HBM = 6650.0  # GB/s, B200_PROFILING.md fallback
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=8)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c5", choices=sorted(ibfs_gen.CONFIGS))
     ap.add_argument("--groups-per-rank", type=int, default=0)

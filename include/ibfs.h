@@ -153,8 +153,24 @@ typedef struct {
   uint32_t groups_in_flight;  /* groups per launch batch; 0 = auto from nv and memory */
   void *cuda_stream;          /* cudaStream_t to launch on; NULL = legacy default stream */
   uint32_t timing;            /* 1: CUDA events around every level kernel -> stats */
-  uint32_t reserved[7];
+  /* Per-instance direction inside a bottom-up level (never changes results).  The paper
+     runs one direction per group; a BU level stops early at a vertex only
+     once every active instance's bit is found there, so one instance with a tiny
+     frontier (a slow source, a small component) turns every row scan into a full one.
+     IBFS_SPLIT_AUTO: in a BU level, the instances whose sampled frontier edge count m_f(j)
+     satisfies m_f(j) * split_div < m_u(j) (their unexplored edges; Beamer's rule per
+     instance) run top-down in the same launch. */
+  uint32_t split;             /* IBFS_SPLIT_* (default AUTO) */
+  uint32_t split_mod;         /* IBFS_SPLIT_FORCE: instances j with j % split_mod == 0 */
+  float split_div;            /* IBFS_SPLIT_AUTO ratio (default 64) */
+  uint32_t reserved[4];
 } ibfs_run_opts;
+
+enum {
+  IBFS_SPLIT_AUTO = 0,   /* small-frontier instances of a BU level run top-down */
+  IBFS_SPLIT_OFF = 1,    /* one direction per group per level, as in the paper */
+  IBFS_SPLIT_FORCE = 2   /* tests: instances j % split_mod == 0 top-down in every BU level */
+};
 
 void ibfs_run_opts_default(ibfs_run_opts *o);
 

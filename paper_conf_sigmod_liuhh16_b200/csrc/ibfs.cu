@@ -784,44 +784,14 @@ extern "C" void ibfs_run_opts_default(ibfs_run_opts *o) {
   o->bu_from = 2;
   o->alpha = 4.0f;
   o->beta = 24.0f;
+  o->split = IBFS_SPLIT_AUTO;
+  o->split_mod = 2;
+  o->split_div = 64.0f;
 }
 
 namespace {
 
 constexpr int LEVELS_PER_CHECK = 2;
-
-// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda needed).
-typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
-                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
-                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-EncodeTiledFn encode_tiled_fn() {
-  static EncodeTiledFn fn = [] {
-    void *p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
-        q != cudaDriverEntryPointSuccess) {
-      cudaGetLastError();
-      p = nullptr;
-    }
-    return reinterpret_cast<EncodeTiledFn>(p);
-  }();
-  return fn;
-}
-
-// [rows][nv] int8 rows at `base` (row stride nv bytes) as a 2-D tensor with [W][DV] boxes,
-// 128-byte swizzle (the depth kernel's shared tile layout).  false if unavailable.
-bool encode_rows_map(CUtensorMap *map, void *base, uint32_t nv, uint32_t rows, int W) {
-  EncodeTiledFn fn = encode_tiled_fn();
-  if (!fn || rows == 0) return false;
-  const cuuint64_t dims[2] = {nv, rows};
-  const cuuint64_t strides[1] = {nv};
-  const cuuint32_t box[2] = {(cuuint32_t)DV, (cuuint32_t)W};
-  const cuuint32_t estr[2] = {1, 1};
-  return fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
 
 // Per-thread, per-device cache of CUDA events and a pinned host word buffer: creating
 // them per call (cudaEventCreate, cudaMallocHost) costs far more than a small level.
@@ -960,6 +930,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.pol.beta = o.beta;
   a.pol.nv_active = g->nv_active;
   a.pol.ne = g->ne;
+  a.pol.split = o.split;
+  a.pol.split_mod = std::max<uint32_t>(1, o.split_mod);
+  a.pol.split_div = o.split_div;
   a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
   for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
   uint32_t first_dir = 0;
@@ -983,7 +956,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     a.out = out_dev ? out_depths + (size_t)gb0 * rows_bytes_per_group : staging;
     const uint32_t rows_in_batch = std::min<uint32_t>(Gb * W, n - gb0 * W);
     CK(cudaMemsetAsync(flags, 0, 4, stream));
-    CK(cudaMemsetAsync(d_m, 0, (size_t)G * W * 8, stream));  // m_s accumulates in depth_kernel
+    CK(cudaMemsetAsync(d_m, 0, (size_t)G * W * 8, stream));  // m_s accumulates in ms_kernel
     cudaEvent_t w0 = timer.next(), w1 = timer.next();
     CK(cudaEventRecord(w0, stream));
     {
@@ -1001,23 +974,30 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     }
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
-    // the rows of this batch as a [rows_in_batch][nv] byte tensor for the depth kernel's TMA
-    // stores (first flush, 16-byte aligned rows); otherwise it writes bytes itself
-    CUtensorMap out_map;
-    std::memset(&out_map, 0, sizeof(out_map));
-    const bool tma_ok = (nv % 16 == 0) && (((uintptr_t)a.out & 15) == 0) && encode_rows_map(&out_map, a.out, nv, rows_in_batch, W);
-    auto flush = [&](int l1) {
+    bool batch_iso = false;  // a source of this batch is isolated (its own zero is a fix-up)
+    for (uint32_t r = 0; r < rows_in_batch; ++r) batch_iso |= csources[(size_t)gb0 * W + r] == NO_VERTEX;
+    auto flush = [&](int l1, bool final_flush) {
       cudaEvent_t d0 = nullptr, d1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
-                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * 3 / Gb)));
+                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * 2 / Gb)));
       const int first = flushed < 0 ? 1 : 0;
-      depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(
-          a, flushed + 1, l1, first, d_m, out_map, (first && tma_ok) ? 1 : 0);
-      if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
+      depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
       launches++;
       st.depth_launches++;
       st.depth_bytes += (uint64_t)Gb * nva * (B * (uint64_t)(l1 - flushed)) + (uint64_t)rows_in_batch * nv;
+      if (first && batch_iso) {
+        iso_fix_kernel<T><<<Gb, 128, 0, stream>>>(a);
+        launches++;
+      }
+      if (final_flush) {  // m_s from the final visited words (reading #11)
+        const uint32_t mx = (uint32_t)std::max<uint64_t>(
+            1, std::min<uint64_t>(((uint64_t)nva + BLOCK - 1) / BLOCK, std::max<uint64_t>(1, (uint64_t)g->num_sms * 4 / Gb)));
+        ms_kernel<T><<<dim3(mx, Gb), BLOCK, 0, stream>>>(a, d_m);
+        launches++;
+        st.depth_bytes += (uint64_t)Gb * nva * (B + 4);
+      }
+      if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
       flushed = l1;
     };
     int level = 1;
@@ -1029,7 +1009,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
       for (int l = level; l < lend; ++l) {
         // level l's commit (of level l-1) zeroes slot l % R, which held level l-R: flush it
         // first (levels <= l-2 are committed by then)
-        if (l - (int)R > flushed) flush(l - 2);
+        if (l - (int)R > flushed) flush(l - 2, false);
         cudaEvent_t e0 = nullptr, e1 = nullptr;
         if (o.timing) { e0 = timer.next(); e1 = timer.next(); CK(cudaEventRecord(e0, stream)); }
         int lv = l;
@@ -1056,7 +1036,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         if (h_done[chunk - 2] >= Gb) break;
       }
     }
-    flush(level - 1);  // the rest (each group stops at its own last level)
+    flush(level - 1, true);  // the rest (each group stops at its own last level)
     CK(cudaEventRecord(w1, stream));
     win.push_back({w0, w1});
     // range check (a level-128 discovery means a depth > 127)
@@ -1167,6 +1147,9 @@ extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_
     if (o.direction > 3) fail(IBFS_E_INVALID, "bad direction mode");
     if (o.direction == IBFS_DIR_SCHEDULE && o.schedule_len > 0 && !o.schedule) fail(IBFS_E_INVALID, "schedule is NULL");
     if (!(o.alpha > 0) || !(o.beta > 0)) fail(IBFS_E_INVALID, "alpha and beta must be > 0");
+    if (o.split > IBFS_SPLIT_FORCE) fail(IBFS_E_INVALID, "bad split mode");
+    if (o.split == IBFS_SPLIT_FORCE && o.split_mod == 0) fail(IBFS_E_INVALID, "split_mod must be > 0");
+    if (o.split == IBFS_SPLIT_AUTO && !(o.split_div > 0)) fail(IBFS_E_INVALID, "split_div must be > 0");
     if (stats) {
       if (stats->per_source_m) std::memset(stats->per_source_m, 0, (size_t)n * 8);
       if (stats->per_source_digest) std::memset(stats->per_source_digest, 0, (size_t)n * 8);

@@ -80,6 +80,11 @@ struct GroupCtrl {
   uint32_t done;
   uint32_t arrive;
   uint32_t last_level;
+  // per-instance direction split of a bottom-up level (include/ibfs.h IBFS_SPLIT_*):
+  // td_bits = the active instances expanded top-down in the next level when dir == BU
+  T td_bits;
+  float bitw[WordBits<T>::value];  // sampled degree sum of the new frontier per instance (commit)
+  float cumw[WordBits<T>::value];  // running sum of bitw over the levels so far (visited edges)
 };
 
 struct Policy {
@@ -89,6 +94,8 @@ struct Policy {
   unsigned long long nv_active;  // vertices with degree > 0
   unsigned long long ne;         // CSR entries
   uint32_t sched_len;
+  uint32_t split, split_mod;  // IBFS_SPLIT_*
+  float split_div;
   uint8_t sched[MAXL];  // 0 TD / 1 BU for level l at index l-1
 };
 
@@ -165,6 +172,21 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
   return m;
+}
+
+// 32 x 32 bit transpose across a warp (rows = lanes, columns = bit positions): on return
+// bit i of lane j is bit j of lane i on entry.  Recursive block swap, 5 shuffle stages.
+__device__ __forceinline__ uint32_t warp_transpose32(uint32_t x) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t masks[5] = {0x0000ffffu, 0x00ff00ffu, 0x0f0f0f0fu, 0x33333333u, 0x55555555u};
+#pragma unroll
+  for (int i = 0; i < 5; ++i) {
+    const int s = 16 >> i;
+    const uint32_t m = masks[i];
+    const uint32_t y = __shfl_xor_sync(FULL, x, s);
+    x = (lane & s) ? ((x & ~m) | ((y & ~m) >> s)) : ((x & m) | ((y & m) << s));
+  }
+  return x;
 }
 
 // Warp-aggregated append of this lane's vertex v to queue class cls when pred holds
@@ -266,6 +288,8 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     c.done = done ? 1u : 0u;
     c.arrive = 0;
     c.last_level = done ? 0xffffffffu : 0u;  // done at init: no snapshot was ever written
+    c.td_bits = wzero_value<T>();
+    for (int j = 0; j < W; ++j) c.bitw[j] = c.cumw[j] = 0.f;
     a.ctrl[g] = c;
     if (rows > 0) {
       LevelStat *l1 = ls + 1;
@@ -360,7 +384,7 @@ struct ExpandSmem {  // static part
   uint32_t cnt[2];
   uint32_t item;
   uint32_t flag;
-  uint32_t nitems[3][MAX_G + 1];     // per class group (heavy / light) item prefix
+  uint32_t pre[3 * MAX_G * 2 + 1];   // item prefix over (phase, group, direction)
   unsigned long long acc[MAX_G][5];  // jfq, fq, proc, insp, writes
 };
 
@@ -445,22 +469,24 @@ __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq
 // the entries are staged in shared memory, then an edge-balanced sweep (load-balanced
 // search on the degree prefix) ORs each frontier word into its unvisited neighbours
 // (Alg. 1 l.4-5): consecutive threads read consecutive adjacency entries.
+// fmask: the instances expanded top-down (all of them in a TD level, td_bits in a split
+// BU level); entries whose frontier word has none of them sweep no edges.
 template <typename T>
 __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq, int g, int cls,
-                        uint32_t i0, uint32_t i1, int level) {
+                        uint32_t i0, uint32_t i1, int level, bool filt, T fmask) {
   const int tid = threadIdx.x;
   const T *F = frontier_buf(a, g, level);
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
-  const bool filt = a.ctrl[g].td_filter != 0;
   const uint32_t *q = queue_of(a, g, cls);
   const uint32_t qn = i1 - i0;
   uint32_t insp = 0, writes = 0;
   for (uint32_t i = tid; i < qn; i += BLOCK) {
     const uint32_t v = queue_at(a, q, cls, i0 + i);
+    const T f = wand(ldg(F + v), fmask);
     tq.start[i] = __ldg(a.off + v);
-    tq.word[i] = ldg(F + v);
-    tq.aux[i] = __ldg(a.deg + v);
+    tq.word[i] = f;
+    tq.aux[i] = wzero(f) ? 0u : __ldg(a.deg + v);
   }
   __syncthreads();
   block_exclusive_scan(tq.aux, qn, sm.wsum);
@@ -508,8 +534,11 @@ struct BuRing {  // per-warp rings of QL / NWARP entries, carved from TileQueue 
 };
 
 template <typename T>
+// active: the group's active instances (Eq. 1 counters, reading #23); td_bits: those a
+// split level expands top-down instead (excluded from T; N[f] is then shared with the
+// top-down part, so the result is ORed in rather than stored).
 __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq, int g, int cls,
-                        uint32_t i0, uint32_t i1, int level, T active) {
+                        uint32_t i0, uint32_t i1, int level, T active, T td_bits) {
   constexpr int QW = QL / NWARP;  // ring entries per warp (128)
   static_assert(sizeof(BuRing<T>) <= sizeof(TileQueue<T>), "BU ring must fit the item storage");
   BuRing<T> &bq = *reinterpret_cast<BuRing<T> *>(&tq);
@@ -518,6 +547,7 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
   const T *vis = a.visited + (size_t)g * a.gstride;
   const uint32_t *q = queue_of(a, g, cls);
   uint32_t jfq = 0, fq = 0, proc = 0, insp = 0, writes = 0;
+  const bool split = !wzero(td_bits);
   if (tid == 0) sm.cnt[0] = i0;
   __syncthreads();
   const int qbase = warp * QW;
@@ -552,9 +582,10 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       if (c_next >= i1) {
         range_done = true;
       } else {
-        const T tx = tx_next;
+        const T tfull = tx_next;
+        const T tx = wandn(tfull, td_bits);
         const bool keep = !wzero(tx);
-        if (keep && level > 1) { jfq++; fq += wpopc(tx); }  // level 1: closed form (init)
+        if (!wzero(tfull) && level > 1) { jfq++; fq += wpopc(tfull); }  // level 1: closed form (init)
         const uint32_t bal = __ballot_sync(FULL, keep);
         if (keep) {
           const uint32_t pos = qbase + ((tail + __popc(bal & lanemask_lt())) & (QW - 1));
@@ -607,7 +638,10 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       for (int u = 0; u < 4; ++u)
         if (w[u] != 0xffffffffu) { acc = wor(acc, wand(x[u], tg)); insp++; }
       if (weq(acc, tg) || k >= d) {
-        if (!wzero(acc)) { st(N + v, acc); writes++; }
+        if (!wzero(acc)) {
+          if (split) red_or(N + v, acc); else st(N + v, acc);
+          writes++;
+        }
         has = false;
       }
     }
@@ -617,14 +651,14 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
 
 // Hub chunk, top-down: CHUNK edges of one hub's row swept by the whole CTA.
 template <typename T>
-__device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubChunk c, int level) {
+__device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubChunk c, int level, bool filt,
+                       T fmask) {
   const int tid = threadIdx.x;
   const T *F = frontier_buf(a, g, level);
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
-  const T f = ldg(F + c.v);
+  const T f = wand(ldg(F + c.v), fmask);
   if (wzero(f)) return;
-  const bool filt = a.ctrl[g].td_filter != 0;
   uint32_t insp = 0, writes = 0;
   constexpr int U = 8;
   for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
@@ -652,13 +686,18 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
 // already found (atomically accumulated in N[hub]).
 template <typename T>
 __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, const HubChunk c,
-                       int level, T active) {
+                       int level, T active, T td_bits) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
-  const T tg = wandn(active, ldg(vis + c.v));
-  if (wzero(tg)) return;
+  const T tfull = wandn(active, ldg(vis + c.v));
+  const T tg = wandn(tfull, td_bits);
   const bool first = c.first && tid == 0;
+  const bool cnt = first && level > 1 && !wzero(tfull);  // level 1: closed form (init)
+  if (wzero(tg)) {
+    flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tfull) : 0u, 0u, 0u, 0u);
+    return;
+  }
   if (tid == 0) sm.flag = weq(wand(ldv(N + c.v), tg), tg) ? 1u : 0u;
   __syncthreads();
   uint32_t insp = 0, writes = 0;
@@ -687,41 +726,46 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
     }
     if (tid == 0 && !wzero(acc)) { red_or(N + c.v, acc); writes++; }
   }
-  const bool cnt = first && level > 1;  // level 1: closed form (init)
-  flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tg) : 0u, first ? 1u : 0u, insp, writes);
+  flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tfull) : 0u, first ? 1u : 0u, insp, writes);
 }
 
 // Expand phase of level `level` for all groups of a batch.  Work items, pulled by CTAs
-// from a per-level counter: frontier hub chunks first, then heavy-queue items, then
-// light-queue items, each carrying its group (whose direction the commit decided).
+// from a per-level counter, in three phases -- frontier hub chunks, then heavy-queue
+// items, then light-queue items -- each carrying its group and direction.  A group runs
+// its top-down part when its level is TD or a split BU level (td_bits != 0), and its
+// bottom-up part when the level is BU.  The control words were written by the commit
+// phase of this launch (before the grid barrier): read them through L2 (ld.cg).
 template <typename T>
 __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T *s_red, TileQueue<T> &tq) {
   const int tid = threadIdx.x;
   for (int i = tid; i < a.G * 5; i += BLOCK) sm.acc[i / 5][i % 5] = 0ull;
   const int par = (level - 1) & 1;  // queues were produced by commit l-1 (or init)
-  if (tid == 0) {
-    uint32_t ph = 0, pl = 0, pc = 0;
-    for (int g = 0; g < a.G; ++g) {
-      const GroupCtrl<T> &c = a.ctrl[g];
-      sm.nitems[0][g] = ph;
-      sm.nitems[1][g] = pl;
-      sm.nitems[2][g] = pc;
-      if (!c.done) {
-        const int base = c.dir ? Q_BUL : Q_TDL;
-        const uint32_t qh = c.dir ? QBH : QH;
-        ph += (c.qlen[par][base + 1] + qh - 1) / qh;
-        pl += (c.qlen[par][base] + QL - 1) / QL;
-        pc += c.qlen[par][c.dir ? Q_BUC : Q_TDC];
+  const int nslot = 3 * a.G * 2;
+  for (int i = tid; i < nslot; i += BLOCK) {  // items of slot (phase, group, direction)
+    const int ph = i / (2 * a.G), g = (i >> 1) % a.G, d = i & 1;
+    const GroupCtrl<T> *c = a.ctrl + g;
+    uint32_t n = 0;
+    if (!ldcg(&c->done)) {
+      const uint32_t dir = ldcg(&c->dir);
+      const bool on = d ? dir == 1 : (dir == 0 || !wzero(ldcg_w(&c->td_bits)));
+      if (on) {
+        const int base = d ? Q_BUL : Q_TDL;
+        const uint32_t *ql = c->qlen[par];
+        if (ph == 0) n = ldcg(ql + (d ? Q_BUC : Q_TDC));
+        else if (ph == 1) { const uint32_t per = d ? QBH : QH; n = (ldcg(ql + base + 1) + per - 1) / per; }
+        else n = (ldcg(ql + base) + QL - 1) / QL;
       }
     }
-    sm.nitems[0][a.G] = ph;
-    sm.nitems[1][a.G] = pl;
-    sm.nitems[2][a.G] = pc;
+    sm.pre[i] = n;
   }
   __syncthreads();
-  const uint32_t n_hub = sm.nitems[2][a.G];
-  const uint32_t n_heavy = sm.nitems[0][a.G];
-  const uint32_t total = n_hub + n_heavy + sm.nitems[1][a.G];
+  if (tid == 0) {  // exclusive prefix (<= 384 slots)
+    uint32_t run = 0;
+    for (int i = 0; i < nslot; ++i) { const uint32_t x = sm.pre[i]; sm.pre[i] = run; run += x; }
+    sm.pre[nslot] = run;
+  }
+  __syncthreads();
+  const uint32_t total = sm.pre[nslot];
   uint32_t pending = 0;
   if (tid == 0) pending = atomicAdd(a.work_ctr + level, 1u);
   for (;;) {
@@ -733,29 +777,31 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     __syncthreads();
     const uint32_t item = sm.item;
     if (item >= total) break;
-    if (item < n_hub) {
-      int g = 0;
-      while (g + 1 < a.G && sm.nitems[2][g + 1] <= item) ++g;
-      const GroupCtrl<T> *c = a.ctrl + g;
-      const uint32_t k = item - sm.nitems[2][g];
-      const HubChunk hc = a.chunks[a.chq[((size_t)g * 2 + (c->dir ? 1 : 0)) * a.n_chunks + k]];
-      if (c->dir == 0) hub_td<T>(a, sm, g, hc, level);
-      else hub_bu<T>(a, sm, s_red, g, hc, level, c->active);
+    uint32_t lo = 0, hi = (uint32_t)nslot;  // the slot with pre[lo] <= item < pre[lo + 1]
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (sm.pre[mid] <= item) lo = mid; else hi = mid;
+    }
+    const int ph = (int)lo / (2 * a.G), g = (int)(lo >> 1) % a.G, d = (int)(lo & 1);
+    const uint32_t k = item - sm.pre[lo];
+    const GroupCtrl<T> *c = a.ctrl + g;
+    const bool bu_level = ldcg(&c->dir) == 1;
+    const T td_bits = bu_level ? ldcg_w(&c->td_bits) : wzero_value<T>();
+    const T all = wnot(wzero_value<T>());
+    const bool filt = ldcg(&c->td_filter) != 0;
+    if (ph == 0) {
+      const HubChunk hc = a.chunks[a.chq[((size_t)g * 2 + d) * a.n_chunks + k]];
+      if (d == 0) hub_td<T>(a, sm, g, hc, level, filt, bu_level ? td_bits : all);
+      else hub_bu<T>(a, sm, s_red, g, hc, level, ldcg_w(&c->active), td_bits);
       continue;
     }
-    const bool heavy = item < n_hub + n_heavy;
-    const int sel = heavy ? 0 : 1;
-    const uint32_t r = heavy ? item - n_hub : item - n_hub - n_heavy;
-    int g = 0;
-    while (g + 1 < a.G && sm.nitems[sel][g + 1] <= r) ++g;
-    const GroupCtrl<T> *c = a.ctrl + g;
-    const uint32_t k = r - sm.nitems[sel][g];
-    const int cls = (c->dir ? Q_BUL : Q_TDL) + (heavy ? 1 : 0);
-    const uint32_t qlen = c->qlen[par][cls];
-    const uint32_t per = c->dir ? (heavy ? QBH : QL) : (heavy ? QH : QL);
+    const bool heavy = ph == 1;
+    const int cls = (d ? Q_BUL : Q_TDL) + (heavy ? 1 : 0);
+    const uint32_t qlen = ldcg(c->qlen[par] + cls);
+    const uint32_t per = d ? (heavy ? QBH : QL) : (heavy ? QH : QL);
     const uint32_t i0 = k * per, i1 = min(qlen, i0 + per);
-    if (c->dir == 0) item_td<T>(a, sm, tq, g, cls, i0, i1, level);
-    else item_bu<T>(a, sm, tq, g, cls, i0, i1, level, c->active);
+    if (d == 0) item_td<T>(a, sm, tq, g, cls, i0, i1, level, filt, bu_level ? td_bits : all);
+    else item_bu<T>(a, sm, tq, g, cls, i0, i1, level, ldcg_w(&c->active), td_bits);
   }
   __syncthreads();
   for (int i = tid; i < a.G; i += BLOCK) {
@@ -803,7 +849,16 @@ struct CommitSmem {
   uint32_t last;
   uint32_t wcnt[NWARP][4];
   uint32_t qbase[4];
+  float bcnt[WordBits<T>::value];       // sampled per-instance frontier degree sums of this CTA
+  uint32_t tdb[WordBits<T>::value / 32];  // split decision (last CTA of a group)
 };
+
+// Per-instance frontier edge counts m_f(j) for the split decision (IBFS_SPLIT_AUTO) are
+// sampled: the first vertex of each thread in every SAMPLE_TILES-th commit tile, i.e.
+// 1 / SAMPLE of the vertices.  A warp transposes its 32 sampled new-bit words (lane i
+// then holds the mask M of sampled vertices new for instance 32p + i) and weights them
+// by degree through the degree bit planes D_b = ballot(bit b of deg): sum_b popc(M & D_b) << b.
+constexpr int SAMPLE_TILES = 4;
 
 // Commit of level lc for one tile of group g: the CVT * BLOCK vertices from `base`.
 // visited |= S_lc, zero slot lc + 1, build both JFQs of level lc + 1 -- top-down: vertices
@@ -814,11 +869,13 @@ struct CommitSmem {
 // (n_f, m_f, new pairs, OR of new bits) accumulate in the caller's registers.
 constexpr int CVT = 4;
 constexpr int CTILE = CVT * BLOCK;  // vertices per commit tile
+constexpr int SAMPLE = SAMPLE_TILES * CVT;
 
 template <typename T>
 __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, size_t base,
                                             unsigned long long &nf, unsigned long long &mf,
-                                            unsigned long long &newp, T &nacc) {
+                                            unsigned long long &newp, T &nacc, bool sample,
+                                            float (&bc)[WordBits<T>::value / 32]) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   GroupCtrl<T> *c = a.ctrl + g;
   const T active = c->active;
@@ -878,6 +935,20 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
 #pragma unroll
     for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
   }
+  if (sample) {  // block-uniform
+    const uint32_t d0 = wzero(n[0]) ? 0u : dg[0];
+    const uint32_t dmax = __reduce_or_sync(FULL, d0);
+    if (dmax) {
+      const int nb = 32 - __clz(dmax);
+#pragma unroll
+      for (int p = 0; p < WordBits<T>::value / 32; ++p) {
+        const uint32_t m = warp_transpose32(wpiece(n[0], p));
+        unsigned long long sum = 0;
+        for (int b = 0; b < nb; ++b) sum += (unsigned long long)__popc(m & __ballot_sync(FULL, (d0 >> b) & 1u)) << b;
+        bc[p] += (float)sum;
+      }
+    }
+  }
   if (lane == 0)
     for (int cls = 0; cls < 4; ++cls) cm.wcnt[warp][cls] = wc[cls];
   __syncthreads();
@@ -910,11 +981,13 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
 }
 
 // Add one CTA's counters for group g (ntiles tiles) to the group, and if they complete the
-// group's tiles, decide the next level: direction (reading #7), active mask, done.
+// group's tiles, decide the next level: direction (reading #7), the per-instance split of
+// a BU level (include/ibfs.h IBFS_SPLIT_*), active mask, done.
 template <typename T>
 __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, uint32_t ntiles,
                              uint32_t tiles_per_group, unsigned long long nf, unsigned long long mf,
-                             unsigned long long newp, T nacc) {
+                             unsigned long long newp, T nacc, float (&bc)[WordBits<T>::value / 32]) {
+  constexpr int W = WordBits<T>::value;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   GroupCtrl<T> *c = a.ctrl + g;
   if (lc >= 128 && !wzero(nacc)) atomicExch(a.range_err, 1u);  // depth > 127
@@ -926,7 +999,15 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     cm.red[warp][0] = nf; cm.red[warp][1] = mf; cm.red[warp][2] = newp;
     cm.orr[warp] = nacc;
   }
+#pragma unroll
+  for (int p = 0; p < W / 32; ++p)
+    if (bc[p] != 0.f) { atomicAdd(&cm.bcnt[p * 32 + lane], bc[p]); bc[p] = 0.f; }
   __syncthreads();
+  if (tid < W) {
+    const float x = cm.bcnt[tid];
+    if (x != 0.f) atomicAdd(&c->bitw[tid], x);
+    cm.bcnt[tid] = 0.f;
+  }
   if (tid == 0) {
     unsigned long long t0 = 0, t1 = 0, t2 = 0;
     T o = wzero_value<T>();
@@ -938,25 +1019,58 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     if (t1) atomicAdd(&c->m_f, t1);
     if (t2) atomicAdd(&c->newp, t2);
     if (!wzero(o)) red_or(&c->newacc, o);
-    __threadfence();
+  }
+  __threadfence();
+  __syncthreads();
+  if (tid == 0) {
     const uint32_t prev = atomicAdd(&c->arrive, ntiles);
     cm.last = (prev + ntiles == tiles_per_group) ? 1u : 0u;
   }
   __syncthreads();
-  if (cm.last && tid == 0) {
-    __threadfence();
-    const T act = ldv(&c->newacc);
+  if (!cm.last) return;  // block-uniform
+  __threadfence();
+  const T act = ldv(&c->newacc);
+  // split: the active instances to expand top-down if the next level is BU -- Beamer's
+  // rule per instance (reading #7): j stays bottom-up only while its frontier edge count
+  // m_f(j) * split_div exceeds its unexplored edge count m_u(j) = ne - sum of the earlier
+  // frontiers' edges (both sampled); FORCE: j % split_mod == 0
+  if (tid < W / 32) cm.tdb[tid] = 0;
+  __syncthreads();
+  if (tid < W) {
+    const float w = *(volatile float *)&c->bitw[tid];
+    const float cum = *(volatile float *)&c->cumw[tid] + w;
+    c->bitw[tid] = 0.f;
+    c->cumw[tid] = cum;
+    bool small;
+    if (a.pol.split == 2) small = (uint32_t)tid % a.pol.split_mod == 0;
+    else {
+      const double mf = (double)w * SAMPLE, mu = fmax((double)a.pol.ne - (double)cum * SAMPLE, 1.0);
+      small = mf * (double)a.pol.split_div < mu;
+    }
+    if (a.pol.split != 1 && small && ((wpiece(act, tid >> 5) >> (tid & 31)) & 1u))
+      atomicOr(&cm.tdb[tid >> 5], 1u << (tid & 31));
+  }
+  __syncthreads();
+  if (tid == 0) {
     const unsigned long long n_f = ldv(&c->n_f), m_f = ldv(&c->m_f), np = ldv(&c->newp);
     const uint32_t cur = c->dir;
     LevelStat *ls = a.lstat + (size_t)g * MAXL + lc;
     ls->dir = cur + 1;
     ls->newp = np;
     ls->nf = n_f;
-    const bool bu = decide_bu(a.pol, (uint32_t)lc + 1, cur, n_f, m_f);
+    bool bu;
+    T tdb = wzero_value<T>();
+    bu = decide_bu(a.pol, (uint32_t)lc + 1, cur, n_f, m_f);
+    if (bu) {
+      tdb = wfrom_pieces<T>(cm.tdb);
+      // auto: if every active instance is small the level is plain top-down
+      if (a.pol.mode == 0 && weq(tdb, act)) { bu = false; tdb = wzero_value<T>(); }
+    }
     c->active = act;
     c->newacc = wzero_value<T>();
     c->n_f = c->m_f = c->newp = 0;
     c->dir = bu ? 1u : 0u;
+    c->td_bits = tdb;
     // top-down pre-check of visited[w] only once a fair share of the (vertex, active
     // instance) pairs is visited; before that nearly every OR is new and the gather is
     // wasted (the commit masks what an unfiltered OR set twice)
@@ -1043,20 +1157,27 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
     uint32_t ntiles = 0;
     unsigned long long nf = 0, mf = 0, newp = 0;
     T nacc = wzero_value<T>();
+    constexpr int NP = WordBits<T>::value / 32;
+    float bc[NP];
+#pragma unroll
+    for (int p = 0; p < NP; ++p) bc[p] = 0.f;
+    for (int j = tid; j < WordBits<T>::value; j += BLOCK) cm.bcnt[j] = 0.f;
+    __syncthreads();
     for (size_t w = blockIdx.x; w < total; w += gridDim.x) {
       const int g = (int)(w / tpg);
       if (g != cur_g) {
-        if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc);
+        if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc);
         cur_g = g;
         ntiles = 0;
         nf = mf = newp = 0;
         nacc = wzero_value<T>();
       }
       if (a.ctrl[g].done) continue;  // finished before this launch (stable)
-      commit_tile(a, cm, g, lc, (size_t)(w % tpg) * CTILE, nf, mf, newp, nacc);
+      const uint32_t tix = (uint32_t)(w % tpg);
+      commit_tile(a, cm, g, lc, (size_t)tix * CTILE, nf, mf, newp, nacc, tix % SAMPLE_TILES == 0, bc);
       ++ntiles;
     }
-    if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc);
+    if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc);
     grid_barrier(a.gbar);
   }
   if (tid == 0 && blockIdx.x == 0) {
@@ -1077,35 +1198,37 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
 // Depth rows from the level snapshots l in [l0, l1] (l1 capped at the group's last
 // committed level and at 127): depth[j][v] = the first l with bit j of S_l[v] set.
 //
-// A CTA owns a tile of DV = 128 consecutive caller-id vertices (columns) x all W rows,
-// staged in a shared [W][128] byte tile (128-byte swizzled, double-buffered) prefilled
-// with -1 (isolated vertices own no snapshot word).  The tile's vertices of degree > 0 are
-// one contiguous range [c0, c0 + k) of compacted ids, so each level's words for the tile
-// are one contiguous run: a producer warp fetches them with 1-D TMA bulk copies
-// (cp.async.bulk, DLB levels per stage, DNS stages on mbarriers), DNS - 1 jobs ahead of
-// the consumers, across tile boundaries.  Consumers are dealt densely over the k
-// vertices (no lane idles on an isolated column): thread t owns vertex slots t%64 and
-// t%64 + 64 for the W/2 instances of half t/64, and accumulates (l + 1) into the byte of
-// every row whose bit first appears at level l (SIMD within a register: bytes never
-// carry, each receives at most one value <= 128).  An isolated source gets 0 in its own
-// row.  The finished tile leaves with one 2-D TMA tensor store (cp.async.bulk.tensor,
-// full 128-byte rows) while the CTA fills the other buffer.  first != 0 writes every
-// byte; otherwise (a ring-slot flush before reuse) only the bytes found in [l0, l1]
-// change, with plain byte stores.
-constexpr int DV = 128;         // columns per tile (= the 128-byte swizzle span)
-constexpr int DTHREADS = 128;   // consumer threads (+ one producer warp)
-constexpr int DLB = 4;          // levels per pipeline stage
-constexpr int DNS = 4;          // pipeline stages (DNS - 1 jobs in flight)
-constexpr int DSLOTS = DTHREADS / 2;  // vertex slots per pass (two halves per vertex)
+// A CTA works through tiles of DV = 128 consecutive caller-id vertices (columns) x all W
+// rows.  The tile's vertices of degree > 0 are one contiguous range [c0, c0 + k) of
+// compacted ids, so each level's words for the tile are one contiguous run: a producer
+// warp fetches them with 1-D TMA bulk copies (cp.async.bulk, up to DLB levels per stage,
+// DNS stages on mbarriers), DNS - 1 tiles ahead of the consumers.
+//   phase A (accumulate): the k words of a level are dealt densely -- consumer thread t
+//     owns dense slot t % 64 (+ 64 in a second round when k > 64) for the W/4 instances
+//     of part t / 64, so no lane idles on an isolated column -- and accumulates (l + 1)
+//     into the byte of every instance whose bit first appears at level l (SIMD within a
+//     register: bytes never carry, each receives at most one value <= 128).  The column
+//     bytes go to a column-major staging tile in shared memory (16-byte chunks, XOR
+//     swizzled by column).
+//   phase B (store): thread t takes column t % 128 in caller order for the W/2
+//     instances of half t / 128 (isolated columns: all -1), turns l + 1 into l (0 -> -1),
+//     and a 4 x 4 byte transpose among the 4 lanes of consecutive columns (2 shuffles + 2
+//     byte permutes per word) gives each lane 4 consecutive columns of one row: a warp
+//     stores 4 rows x 32 contiguous bytes per instruction (full 32-byte sectors,
+//     streaming stores -- the rows are written once and not re-read here).
+// first != 0 writes every byte; otherwise (a ring-slot flush before reuse) only the bytes
+// found in [l0, l1] change.  m_s and the isolated sources' own zero are separate passes.
+constexpr int DV = 128;               // columns per tile
+constexpr int DCW = 8;                // consumer warps
+constexpr int DTHREADS = DCW * 32;    // consumer threads
+constexpr int DSLOTS = 64;            // dense slots per round (DTHREADS / 4 parts)
+constexpr int DLB = 10;               // levels per pipeline stage
+constexpr int DNS = 3;                // pipeline stages
+constexpr int DHDR = 32 + DV;         // stage header: k, run offset, c0, pad, nzbits[4]; slot -> column table
 
 __device__ __forceinline__ uint32_t spread4(uint32_t nib) {
   // 4-bit nibble -> 0x01 in each byte whose bit is set
   return (nib * 0x00204081u) & 0x01010101u;
-}
-
-// byte offset of (row r, column c) in a 128-byte-swizzled [rows][128] tile
-__device__ __forceinline__ uint32_t sw128(uint32_t r, uint32_t c) {
-  return r * 128u + ((((c >> 4) ^ r) & 7u) << 4) + (c & 15u);
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -1120,77 +1243,73 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(unsigned long long *bar, u
 __device__ __forceinline__ void mbar_arrive(unsigned long long *bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+// Wait for phase `parity` to complete; the thread is suspended inside try_wait (time
+// hint) instead of spinning on the issue slots.
 __device__ __forceinline__ void mbar_wait(unsigned long long *bar, uint32_t parity) {
   asm volatile(
       "{\n .reg .pred p;\n WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
       " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
+      "r"(parity), "r"(1000000u)
       : "memory");
 }
 // 1-D TMA bulk copy global -> shared (16-byte aligned, size a multiple of 16), completing
 // `bytes` of transaction count on the mbarrier.
-__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, unsigned long long *bar) {
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, unsigned long long *bar) {
   asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(dst)),
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
-// 2-D TMA tensor store shared -> global of one box at (x, y), as a bulk group.
-__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, const void *src, int x, int y) {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(map), "r"(x),
-               "r"(y), "r"(smem_u32(src))
-               : "memory");
-  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-}
-__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
-__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
 // barrier among the DTHREADS consumer threads only (the producer warp never joins)
 __device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(DTHREADS) : "memory"); }
 
-// m16n8k32 u8 x u8 -> s32 tensor-core MMA (D += A * B), fragments per the PTX ISA.
-__device__ __forceinline__ void mma_u8_m16n8k32(int (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2,
-                                                uint32_t a3, uint32_t b0, uint32_t b1) {
-  asm volatile(
-      "mma.sync.aligned.m16n8k32.row.col.s32.u8.u8.s32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
-      "{%0,%1,%2,%3};\n"
-      : "+r"(d[0]), "+r"(d[1]), "+r"(d[2]), "+r"(d[3])
-      : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+// explicit shared-space accesses (32-bit shared addresses)
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds16(uint32_t a) {
+  unsigned short v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds8(uint32_t a) {
+  unsigned short v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) { asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v)); }
+__device__ __forceinline__ void sts64(uint32_t a, uint32_t x, uint32_t y) {
+  asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(a), "r"(x), "r"(y));
+}
+__device__ __forceinline__ void sts128(uint32_t a, uint32_t x, uint32_t y, uint32_t z, uint32_t w) {
+  asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(x), "r"(y), "r"(z), "r"(w));
 }
 
-// byte b of four consecutive degrees, packed little-endian
-__device__ __forceinline__ uint32_t byte_plane4(const uint32_t *d, int b) {
-  const int sh = 8 * b;
-  return ((d[0] >> sh) & 0xffu) | (((d[1] >> sh) & 0xffu) << 8) | (((d[2] >> sh) & 0xffu) << 16) |
-         (((d[3] >> sh) & 0xffu) << 24);
-}
-
-// add the MMA accumulators (rows 0..3 = byte planes; lanes with gq < 4) into s_m, reset
-template <int NT>
-__device__ __forceinline__ void flush_macc(int (&dacc)[NT][4], unsigned long long *s_m, int warp, int gq,
-                                           int tq4) {
-  if (gq < 4) {
-#pragma unroll
-    for (int nt = 0; nt < NT; ++nt) {
-      const int j0 = (warp * NT + nt) * 8 + tq4 * 2;
-      if (dacc[nt][0]) atomicAdd(&s_m[j0], (unsigned long long)(uint32_t)dacc[nt][0] << (8 * gq));
-      if (dacc[nt][1]) atomicAdd(&s_m[j0 + 1], (unsigned long long)(uint32_t)dacc[nt][1] << (8 * gq));
-    }
-  }
-#pragma unroll
-  for (int nt = 0; nt < NT; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
+// the W/4-bit part p of a status word at shared address a (little-endian pieces)
+template <int PB>
+__device__ __forceinline__ uint32_t lds_part(uint32_t a) {
+  if (PB == 32) return lds32(a);
+  if (PB == 16) return lds16(a);
+  return lds8(a);
 }
 
 template <typename T>
 struct DepthLayout {
   static constexpr int W = WordBits<T>::value;
-  static constexpr size_t TILE = (size_t)W * DV;                     // one output buffer
+  static constexpr size_t COLB = (size_t)DV * W;                     // one column-major staging tile
   static constexpr size_t SROW = (size_t)DV * sizeof(T) + 16;        // one level's run (+ slack)
-  static constexpr size_t STAGE = DLB * SROW;
-  static constexpr size_t BYTES = 1024 + 2 * TILE + DNS * STAGE;     // + 1024 for alignment
+  static constexpr size_t STAGE = DHDR + DLB * SROW;
+  static constexpr size_t BYTES = 128 + 2 * COLB + DNS * STAGE;      // + 128 for alignment
+  static_assert(DHDR % 16 == 0 && SROW % 16 == 0 && STAGE % 16 == 0, "stage runs must stay 16-byte aligned");
 };
 
 template <typename T>
@@ -1198,253 +1317,282 @@ constexpr size_t depth_smem_bytes() {
   return DepthLayout<T>::BYTES;
 }
 
-// column (within the tile) of the i-th vertex of degree > 0, from the tile's 4 nzbits words
-__device__ __forceinline__ int dense_col(uint4 w, uint32_t p0, uint32_t p1, uint32_t p2, uint32_t i) {
-  if (i < p0) return (int)__fns(w.x, 0, i + 1);
-  if (i < p1) return 32 + (int)__fns(w.y, 0, i - p0 + 1);
-  if (i < p2) return 64 + (int)__fns(w.z, 0, i - p1 + 1);
-  return 96 + (int)__fns(w.w, 0, i - p2 + 1);
+// byte offset of chunk `ch` (16 bytes) of column `col` in a column-major staging tile
+template <int W>
+__device__ __forceinline__ uint32_t colb_off(uint32_t col, uint32_t ch) {
+  constexpr uint32_t NCH = W / 16;  // chunks per column
+  return col * (uint32_t)W + ((ch ^ (col & (NCH - 1))) << 4);
 }
 
-// The same pass accumulates m_s (reading #11): every byte it finds adds deg(v) to row j's
-// sum (each (j, v) is found in exactly one flush) -- a [4 x DV] x [DV x W] u8 product per
-// tile on the tensor cores, flushed to m_out once per CTA.
-//
-// Warp roles: warps 0 .. DTHREADS/32 - 1 consume; the last warp produces (one lane issues
-// the bulk copies).  Stage st is "full" when its bytes landed (s_full[st], expect_tx) and
-// "empty" when every consumer warp has read it (s_empty[st], one arrive per warp).
+// Warp roles: warps 0 .. DCW - 1 consume; warp DCW produces (all lanes write the header's
+// dense slot -> column table, lane 0 issues the copies).  Stage st is "full" when the 32
+// producer lanes arrived and its bytes landed (s_full[st], one expect_tx), "empty" when
+// every consumer warp has read it (s_empty[st]).
 template <typename T>
-__global__ void __launch_bounds__(DTHREADS + 32, 3)
-    depth_kernel(BatchArgs<T> a, int l0, int l1, int first, unsigned long long *m_out,
-                 const __grid_constant__ CUtensorMap out_map, int use_tma) {
+__global__ void __launch_bounds__(DTHREADS + 32, 2)
+    depth_kernel(BatchArgs<T> a, int l0, int l1, int first) {
   using L = DepthLayout<T>;
   constexpr int W = WordBits<T>::value;
-  constexpr int HQ = W / 8;                        // 32-bit byte registers per (vertex, half)
-  constexpr int NWD = DTHREADS / 32;               // consumer warps
-  constexpr int NTILES = W / 8;                    // 8-row n-tiles of the MMA
-  constexpr int NTW = NTILES >= NWD ? NTILES / NWD : 1;
-  constexpr int MMA_WARPS = NTILES / NTW;          // warps taking part in the MMA
+  constexpr int PB = W / 4;        // instances per part (phase A)
+  constexpr int PQ = PB / 4;       // byte registers per part
+  constexpr int HW = W / 8;        // byte registers per half column (phase B)
+  constexpr int NCH = W / 16;      // 16-byte chunks per column
   extern __shared__ unsigned char dsm_raw[];
-  unsigned char *dsm = reinterpret_cast<unsigned char *>(((uintptr_t)dsm_raw + 1023) & ~(uintptr_t)1023);
-  unsigned char *tiles = dsm;                          // [2][W][128], 128B-swizzled
-  unsigned char *stage_base = dsm + 2 * L::TILE;       // [DNS][DLB][SROW]
+  const uint32_t sbase = (smem_u32(dsm_raw) + 127u) & ~127u;
+  const uint32_t colb = sbase;                   // [2][DV][W] column-major staging
+  const uint32_t stage_base = sbase + 2 * (uint32_t)L::COLB;
   __shared__ __align__(8) unsigned long long s_full[DNS], s_empty[DNS];
-  __shared__ uint32_t s_deg[DV];
-  __shared__ unsigned long long s_m[W];
-  __shared__ uint32_t s_isrc[W];  // caller id of row j's source if it is isolated, else NO_VERTEX
-  __shared__ uint32_t s_has_iso;
-  __shared__ uint32_t s_stage_off[DNS];  // byte offset of element 0 inside each stage row
   const int g = blockIdx.y;
   const int rows = group_rows(a, g);
   if (rows == 0) return;
   const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
-  const int gq = lane >> 2, tq4 = lane & 3;  // mma fragment coordinates
-  const int slot = t % DSLOTS, half = t / DSLOTS;
   const GroupCtrl<T> *c = a.ctrl + g;
   const int last = min((int)c->last_level, min(l1, 127));
   const int nlev = last - l0 + 1;  // levels to read (may be <= 0)
-  const int nbat = nlev > 0 ? (nlev + DLB - 1) / DLB : 0;
-  int8_t *out = a.out + (size_t)g * W * a.nv;
+  if (nlev <= 0 && !first) return;
+  const int nbat = nlev > 0 ? (nlev + DLB - 1) / DLB : 1;  // >= 1 job per tile (its header)
   const size_t nvv = a.nv;
   const size_t ntiles = (nvv + DV - 1) / DV;
   const size_t my_tiles = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
   const size_t njobs = my_tiles * (size_t)nbat;
   if (t == 0) {
-    s_has_iso = 0;
     for (int k = 0; k < DNS; ++k) {
-      mbar_init(&s_full[k], 1);
-      mbar_init(&s_empty[k], NWD);
+      mbar_init(&s_full[k], 32);
+      mbar_init(&s_empty[k], DCW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (warp == NWD) {
+  if (warp == DCW) {
     // ---- producer: job jb = (tile jb / nbat of this CTA, batch jb % nbat) -> stage jb % DNS
-    if (lane == 0 && njobs) {
-      uint32_t c0n = __ldg(a.tbase + blockIdx.x), c1n = __ldg(a.tbase + blockIdx.x + 1);
-      uint32_t c0 = 0, k = 0;
-      for (size_t jb = 0; jb < njobs; ++jb) {
-        const int st = (int)(jb % DNS);
-        const int b = (int)(jb % nbat);
-        if (b == 0) {  // a new tile: take its prefetched range, prefetch the next tile's
-          c0 = c0n;
-          k = c1n - c0n;
-          const size_t nt = blockIdx.x + (jb / nbat + 1) * gridDim.x;
-          if (nt < ntiles) {
-            c0n = __ldg(a.tbase + nt);
-            c1n = __ldg(a.tbase + nt + 1);
-          }
-        }
-        if (jb >= (size_t)DNS) mbar_wait(&s_empty[st], (uint32_t)((jb / DNS - 1) & 1));
-        const int lb = l0 + b * DLB, le = min(last, lb + DLB - 1);
-        uint32_t total = 0, off = 0, size = 0;
-        if (k) {
-          const uintptr_t src0 = (uintptr_t)(snap(a, g, lb) + c0);
-          off = (uint32_t)(src0 & 15u);
-          size = (uint32_t)((off + (size_t)k * sizeof(T) + 15) & ~(size_t)15);
-          total = size * (uint32_t)(le - lb + 1);
-        }
-        s_stage_off[st] = off;
-        mbar_arrive_expect_tx(&s_full[st], total);
-        if (k)
-          for (int l = lb; l <= le; ++l) {
-            const unsigned char *src = reinterpret_cast<const unsigned char *>(snap(a, g, l) + c0) - off;
-            bulk_g2s(stage_base + (size_t)st * L::STAGE + (size_t)(l - lb) * L::SROW, src, size, &s_full[st]);
-          }
+    for (size_t jb = 0; jb < njobs; ++jb) {
+      const int st = (int)(jb % DNS);
+      const int b = (int)(jb % nbat);
+      const size_t tix = blockIdx.x + (jb / nbat) * gridDim.x;
+      const uint32_t c0 = __ldg(a.tbase + tix), k = __ldg(a.tbase + tix + 1) - c0;
+      const uint4 nzw = __ldg(reinterpret_cast<const uint4 *>(a.nzbits) + tix);  // bits beyond nv are 0
+      const int lb = l0 + b * DLB, le = min(last, lb + DLB - 1);
+      const int nl = le >= lb ? le - lb + 1 : 0;
+      uint32_t off = 0, size = 0;
+      if (k && nl) {
+        const uintptr_t src0 = (uintptr_t)(snap(a, g, lb) + c0);
+        off = (uint32_t)(src0 & 15u);
+        size = (uint32_t)((off + (size_t)k * sizeof(T) + 15) & ~(size_t)15);
       }
+      if (jb >= (size_t)DNS) mbar_wait(&s_empty[st], (uint32_t)((jb / DNS - 1) & 1));
+      const uint32_t sb = stage_base + (uint32_t)(st * L::STAGE);
+      // dense slot -> column table: lane l places the columns 4l .. 4l + 3 of degree > 0
+      const uint32_t wv = lane < 8 ? nzw.x : lane < 16 ? nzw.y : lane < 24 ? nzw.z : nzw.w;
+      const uint32_t nib = (wv >> (4 * (lane & 7))) & 0xFu;
+      const uint32_t cnt = __popc(nib);
+      uint32_t incl = cnt;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, d);
+        if (lane >= d) incl += y;
+      }
+      uint32_t pos = incl - cnt;
+#pragma unroll
+      for (int cc = 0; cc < 4; ++cc)
+        if ((nib >> cc) & 1u) {
+          asm volatile("st.shared.u8 [%0], %1;" ::"r"(sb + 32 + pos), "h"((unsigned short)(4 * lane + cc)));
+          ++pos;
+        }
+      if (lane == 0) {
+        sts128(sb, k, off, c0, 0u);
+        sts128(sb + 16, nzw.x, nzw.y, nzw.z, nzw.w);
+      }
+      const uint32_t total = size * (uint32_t)nl;
+      if (lane == 0) mbar_arrive_expect_tx(&s_full[st], total); else mbar_arrive(&s_full[st]);
+      if (lane == 0)
+        for (int l = lb; l <= le && total; ++l) {
+          const unsigned char *src = reinterpret_cast<const unsigned char *>(snap(a, g, l) + c0) - off;
+          bulk_g2s(sb + DHDR + (uint32_t)((l - lb) * L::SROW), src, size, &s_full[st]);
+        }
     }
   } else {
     // ---- consumers
-    int dacc[NTW][4];
-#pragma unroll
-    for (int nt = 0; nt < NTW; ++nt) dacc[nt][0] = dacc[nt][1] = dacc[nt][2] = dacc[nt][3] = 0;
-    int tiles_acc = 0;
-    for (int j = t; j < W; j += DTHREADS) {
-      s_m[j] = 0;
-      uint32_t x = NO_VERTEX;
-      if (j < rows && a.csrc[(size_t)g * W + j] == NO_VERTEX) {
-        x = a.src[(size_t)g * W + j];
-        s_has_iso = 1;
-      }
-      s_isrc[j] = x;
-    }
+    const int part = t / DSLOTS, dslot = t % DSLOTS;      // phase A
+    const int col = t % DV, half = t / DV;                // phase B
+    const int q4 = lane & 3;                               // lane within its column quad
+    const uint32_t sel1 = (q4 & 1) ? 0x3726u : 0x5140u;
+    const uint32_t sel2 = (q4 & 2) ? 0x3276u : 0x5410u;
+    const int rowperm = (q4 == 1) ? 2 : (q4 == 2 ? 1 : q4);  // row held after the transpose
+    const bool word_ok = (nvv % 4) == 0;
     size_t job = 0;
     int buf = 0;
-    // the tile's 4 nzbits words and compacted base, prefetched one tile ahead
-    uint4 nzw_next = blockIdx.x < ntiles ? __ldg(reinterpret_cast<const uint4 *>(a.nzbits) + blockIdx.x) : uint4{};
-    uint32_t c0_next = blockIdx.x < ntiles ? __ldg(a.tbase + blockIdx.x) : 0u;
     for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x, buf ^= 1) {
       const size_t v0 = tix * DV;
-      unsigned char *tb = tiles + (size_t)buf * L::TILE;
-      const uint32_t *tw = reinterpret_cast<const uint32_t *>(tb);
-      const uint4 nzw = nzw_next;  // bits beyond nv are 0
-      const uint32_t c0t = c0_next;
-      if (tix + gridDim.x < ntiles) {
-        nzw_next = __ldg(reinterpret_cast<const uint4 *>(a.nzbits) + tix + gridDim.x);
-        c0_next = __ldg(a.tbase + tix + gridDim.x);
-      }
-      const uint32_t p0 = __popc(nzw.x), p1 = p0 + __popc(nzw.y), p2 = p1 + __popc(nzw.z);
-      const uint32_t kcount = p2 + __popc(nzw.w);
-      uint32_t dgr[2];  // degrees of my two slots, in flight during the level batches
-#pragma unroll
-      for (int r = 0; r < 2; ++r) {
-        const uint32_t i = slot + DSLOTS * r;
-        dgr[r] = (i < kcount && half == 0) ? __ldg(a.deg + c0t + i) : 0u;
-      }
-      if (t == 0 && use_tma) bulk_wait_read1();  // this buffer's previous store has read it out
-      consumers_sync();                          // ... and the previous tile's readers are done
-      s_deg[t] = 0;
-      for (int k4 = t; k4 < (int)(L::TILE / 16); k4 += DTHREADS)
-        reinterpret_cast<int4 *>(tb)[k4] = make_int4(-1, -1, -1, -1);
-      uint32_t acc[2][HQ];
+      const uint32_t cb = colb + (uint32_t)(buf * L::COLB);
+      uint32_t acc[2][PQ];
 #pragma unroll
       for (int r = 0; r < 2; ++r)
 #pragma unroll
-        for (int q = 0; q < HQ; ++q) acc[r][q] = 0;
-      unsigned long long reached[2] = {0ull, 0ull};
+        for (int q = 0; q < PQ; ++q) acc[r][q] = 0;
+      uint32_t reached[2] = {0u, 0u};
+      uint32_t k = 0, mynz = 0, dcol[2] = {0u, 0u};
       for (int b = 0; b < nbat; ++b, ++job) {
         const int st = (int)(job % DNS);
         mbar_wait(&s_full[st], (uint32_t)((job / DNS) & 1));
-        const unsigned char *sb = stage_base + (size_t)st * L::STAGE + s_stage_off[st];
+        const uint32_t sb = stage_base + (uint32_t)(st * L::STAGE);
+        const uint32_t off = lds32(sb + 4);
+        if (b == 0) {
+          k = lds32(sb);
+          mynz = (lds32(sb + 16 + 4 * (col >> 5)) >> (col & 31)) & 1u;
+#pragma unroll
+          for (int r = 0; r < 2; ++r) {
+            const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
+            if (i < k) dcol[r] = lds8(sb + 32 + i);
+          }
+        }
         const int lb = l0 + b * DLB, le = min(last, lb + DLB - 1);
 #pragma unroll
         for (int r = 0; r < 2; ++r) {
-          const uint32_t i = slot + DSLOTS * r;
-          if (i < kcount) {
+          const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
+          if (i < k) {
+            const uint32_t p = sb + DHDR + off + i * (uint32_t)sizeof(T) + (uint32_t)(part * PB / 8);
 #pragma unroll
             for (int u = 0; u < DLB; ++u) {
               if (lb + u > le) break;
-              const T wv = *reinterpret_cast<const T *>(sb + (size_t)u * L::SROW + (size_t)i * sizeof(T));
-              const unsigned long long hb = whalf(wv, half) & ~reached[r];
+              const uint32_t hb = lds_part<PB>(p + (uint32_t)(u * L::SROW)) & ~reached[r];
               if (!hb) continue;
-              reached[r] |= hb;
               const uint32_t inc = (uint32_t)(lb + u + 1);
+              if (reached[r] == 0u && hb == (PB == 32 ? 0xffffffffu : ((1u << PB) - 1u))) {
+                // the whole part at one level (common): no bit spreading
 #pragma unroll
-              for (int q = 0; q < HQ; ++q) acc[r][q] += spread4((uint32_t)(hb >> (4 * q)) & 0xFu) * inc;
+                for (int q = 0; q < PQ; ++q) acc[r][q] = inc * 0x01010101u;
+              } else {
+#pragma unroll
+                for (int q = 0; q < PQ; ++q) acc[r][q] += spread4((hb >> (4 * q)) & 0xFu) * inc;
+              }
+              reached[r] |= hb;
             }
           }
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&s_empty[st]);  // this warp is done with stage st
       }
-      consumers_sync();  // prefill done everywhere before the columns land
-      // the tile's columns
+      // phase A -> staging (dense slot i of the tile is column dcol, from the stage table)
 #pragma unroll
       for (int r = 0; r < 2; ++r) {
-        const uint32_t i = slot + DSLOTS * r;
-        if (i < kcount) {
-          const uint32_t col = (uint32_t)dense_col(nzw, p0, p1, p2, i);
-          if (half == 0) s_deg[col] = dgr[r];
-          // swizzled column offset for each row phase (row & 7), so every store below is
-          // base + row * 128 + cs[row & 7] with a compile-time row
-          uint32_t cs[8];
-#pragma unroll
-          for (int k = 0; k < 8; ++k) cs[k] = ((((col >> 4) ^ (uint32_t)k) & 7u) << 4) + (col & 15u);
-          unsigned char *hb = tb + half * (W / 2) * 128;
-#pragma unroll
-          for (int q = 0; q < HQ; ++q) {
-            const uint32_t x = __vsub4(acc[r][q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
-#pragma unroll
-            for (int bb = 0; bb < 4; ++bb) {
-              const int row = q * 4 + bb;  // (half * W/2 is a multiple of 8: same phase)
-              hb[row * 128 + cs[row & 7]] = (unsigned char)(x >> (8 * bb));
-            }
+        const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
+        if (i < k) {
+          const uint32_t dc = dcol[r];
+          const uint32_t byte0 = (uint32_t)(part * PB);  // first instance of the part
+          if (PB == 32) {
+            sts128(cb + colb_off<W>(dc, byte0 / 16), acc[r][0], acc[r][1], acc[r][2], acc[r][3]);
+            sts128(cb + colb_off<W>(dc, byte0 / 16 + 1), acc[r][4 % PQ], acc[r][5 % PQ], acc[r][6 % PQ],
+                   acc[r][7 % PQ]);
+          } else if (PB == 16) {
+            sts128(cb + colb_off<W>(dc, byte0 / 16), acc[r][0], acc[r][1 % PQ], acc[r][2 % PQ], acc[r][3 % PQ]);
+          } else {
+            sts64(cb + colb_off<W>(dc, byte0 / 16) + (byte0 & 15u), acc[r][0], acc[r][1 % PQ]);
           }
         }
       }
-      consumers_sync();
-      if (s_has_iso) {  // isolated sources: depth 0 in their own row (degree 0: no m_s)
-        for (int j = t; j < rows; j += DTHREADS) {
-          const uint32_t s = s_isrc[j];
-          if (s != NO_VERTEX && s >= v0 && s < v0 + DV) tb[sw128(j, s - v0)] = 0;
-        }
-        consumers_sync();
-      }
-      if (use_tma) {
-        if (t == 0) tma_store_2d(&out_map, tb, (int)v0, g * W);
-      } else if (v0 + t < nvv) {
-        for (int j = 0; j < rows; ++j) {
-          const int8_t d = (int8_t)tb[sw128(j, t)];
-          if (first || d != -1) out[(size_t)j * nvv + v0 + t] = d;
-        }
-      }
-      // m_s on the tensor cores: D[b][j] += sum_v deg_b(v) * reached(j, v), deg_b = byte b
-      // of deg(v) (A: 16 x 32 u8, rows 0..3 = byte planes), reached from the tile (B: 32 x
-      // 8 u8, 0/1); m_s[j] = sum_b D[b][j] << 8b.
-      if (kcount && warp < MMA_WARPS) {
+      consumers_sync();  // staging complete (and the previous tile's readers of this buffer are done)
+      // phase B: column `col`, rows half * W/2 .. + W/2 - 1
+      uint32_t x[HW];
+      if (mynz) {
 #pragma unroll
-        for (int ks = 0; ks < DV / 32; ++ks) {
-          uint32_t a0 = 0, a2 = 0;
-          if (gq < 4) {
-            const int vb = ks * 32 + tq4 * 4;
-            a0 = byte_plane4(s_deg + vb, gq);
-            a2 = byte_plane4(s_deg + vb + 16, gq);
-          }
-#pragma unroll
-          for (int nt = 0; nt < NTW; ++nt) {
-            const int j = (warp * NTW + nt) * 8 + gq;
-            const uint32_t w0 = j * 32 + ((((uint32_t)(2 * ks) ^ (uint32_t)j) & 7u) << 2) + tq4;
-            const uint32_t w1 = j * 32 + ((((uint32_t)(2 * ks + 1) ^ (uint32_t)j) & 7u) << 2) + tq4;
-            const uint32_t b0 = __vcmpne4(tw[w0], 0xffffffffu) & 0x01010101u;
-            const uint32_t b1 = __vcmpne4(tw[w1], 0xffffffffu) & 0x01010101u;
-            mma_u8_m16n8k32(dacc[nt], a0, 0u, a2, 0u, b0, b1);
-          }
+        for (int cq = 0; cq < HW / 4; ++cq) {
+          const uint4 v = lds128(cb + colb_off<W>((uint32_t)col, (uint32_t)(half * (NCH / 2) + cq)));
+          x[4 * cq] = v.x; x[4 * cq + 1] = v.y; x[4 * cq + 2] = v.z; x[4 * cq + 3] = v.w;
         }
-        if (++tiles_acc == 4096) {  // int32 headroom: <= DV * 255 per tile and element
-          flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
-          tiles_acc = 0;
+      } else {
+#pragma unroll
+        for (int q = 0; q < HW; ++q) x[q] = 0;
+      }
+      const size_t cbase = v0 + (size_t)(col & ~3);  // first column of this lane's quad
+      const int row0 = half * (W / 2) + rowperm;
+      int8_t *dst = a.out + ((size_t)g * W + row0) * nvv + cbase;  // row row0 + 4q at dst + 4q nv
+      const bool fast = word_ok && v0 + DV <= nvv && first && rows == W;  // block-uniform
+#pragma unroll
+      for (int q = 0; q < HW; ++q, dst += 4 * nvv) {
+        uint32_t w = __vsub4(x[q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
+        uint32_t y = __shfl_xor_sync(FULL, w, 1);
+        w = __byte_perm(w, y, sel1);
+        y = __shfl_xor_sync(FULL, w, 2);
+        w = __byte_perm(w, y, sel2);
+        if (fast) {
+          __stcs(reinterpret_cast<unsigned int *>(dst), w);
+        } else {
+          if (row0 + 4 * q >= rows) continue;
+          const uint32_t ff = __vcmpeq4(w, 0xffffffffu);
+          if (word_ok && v0 + DV <= nvv && ff == 0) {
+            __stcs(reinterpret_cast<unsigned int *>(dst), w);
+          } else {
+#pragma unroll
+            for (int bb = 0; bb < 4; ++bb)
+              if (cbase + bb < nvv && (first || !((ff >> (8 * bb)) & 1u))) dst[bb] = (int8_t)(w >> (8 * bb));
+          }
         }
       }
     }
-    if (warp < MMA_WARPS) flush_macc<NTW>(dacc, s_m, warp, gq, tq4);
-    if (t == 0 && use_tma) bulk_wait_all();
   }
-  __syncthreads();
-  for (int j = t; j < rows; j += DTHREADS)
-    if (s_m[j]) atomicAdd(&m_out[(size_t)g * W + j], s_m[j]);
 }
 
 // --------------------------------------------------------------------- finalize ----
+// m_s (reading #11): m_s[j] = sum_v deg(v) * bit j of visited[v] over
+// the final visited words (compacted ids: isolated vertices have degree 0).  A warp takes
+// 32 vertices at a time: a 32 x 32 bit transpose per 32-bit piece gives lane i the mask
+// M of the warp's vertices reached by instance 32p + i, and the degree-weighted count is
+// sum_b popc(M & D_b) << b over the degree bit planes D_b = ballot(bit b of deg).
+template <typename T>
+__global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long long *m_out) {
+  constexpr int W = WordBits<T>::value;
+  constexpr int NP = W / 32;
+  __shared__ unsigned long long s_m[W];
+  const int g = blockIdx.y;
+  const int rows = group_rows(a, g);
+  // a group finished at init (every source isolated) never zeroed its visited words; its
+  // instances reach nothing of positive degree: m_s = 0
+  if (rows == 0 || a.ctrl[g].last_level == 0xffffffffu) return;
+  const int tid = threadIdx.x, lane = tid & 31;
+  for (int j = tid; j < W; j += BLOCK) s_m[j] = 0;
+  __syncthreads();
+  const T *vis = a.visited + (size_t)g * a.gstride;
+  unsigned long long acc[NP];
+#pragma unroll
+  for (int p = 0; p < NP; ++p) acc[p] = 0;
+  const size_t nvr = ((size_t)a.nva + 31) & ~(size_t)31;  // warp-uniform trip count
+  for (size_t v = (size_t)blockIdx.x * BLOCK + tid; v < nvr; v += (size_t)gridDim.x * BLOCK) {
+    const bool in = v < a.nva;
+    const T x = in ? ldg(vis + v) : wzero_value<T>();
+    const uint32_t d = in ? __ldg(a.deg + v) : 0u;
+    const uint32_t any = __ballot_sync(FULL, !wzero(x) && d != 0);
+    if (!any) continue;
+    uint32_t m[NP];
+#pragma unroll
+    for (int p = 0; p < NP; ++p) m[p] = warp_transpose32(wpiece(x, p));
+    const uint32_t dmax = __reduce_or_sync(FULL, d);
+    const int nb = 32 - __clz(dmax);
+    for (int b = 0; b < nb; ++b) {
+      const uint32_t db = __ballot_sync(FULL, (d >> b) & 1u);
+#pragma unroll
+      for (int p = 0; p < NP; ++p) acc[p] += (unsigned long long)__popc(m[p] & db) << b;
+    }
+  }
+#pragma unroll
+  for (int p = 0; p < NP; ++p)
+    if (acc[p]) atomicAdd(&s_m[p * 32 + lane], acc[p]);
+  __syncthreads();
+  for (int j = tid; j < rows; j += BLOCK)
+    if (s_m[j]) atomicAdd(&m_out[(size_t)g * W + j], s_m[j]);
+}
+
+// Instances whose source is isolated (degree 0) never enter the status words: depth 0 at
+// their own source, after the rows' first flush wrote -1 there.
+template <typename T>
+__global__ void iso_fix_kernel(BatchArgs<T> a) {
+  constexpr int W = WordBits<T>::value;
+  const int g = blockIdx.x;
+  const int rows = group_rows(a, g);
+  for (int j = threadIdx.x; j < rows; j += blockDim.x)
+    if (a.csrc[(size_t)g * W + j] == NO_VERTEX)
+      a.out[((size_t)g * W + j) * a.nv + a.src[(size_t)g * W + j]] = 0;
+}
+
 __device__ __forceinline__ unsigned long long splitmix64(unsigned long long z) {
   z += 0x9E3779B97F4A7C15ull;
   z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;

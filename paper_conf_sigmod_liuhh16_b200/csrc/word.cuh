@@ -30,6 +30,10 @@ __host__ __device__ __forceinline__ uint32_t wandn(uint32_t a, uint32_t b) { ret
 __host__ __device__ __forceinline__ unsigned long long wandn(unsigned long long a, unsigned long long b) { return a & ~b; }
 __host__ __device__ __forceinline__ u128 wandn(u128 a, u128 b) { return {a.lo & ~b.lo, a.hi & ~b.hi}; }
 
+__host__ __device__ __forceinline__ uint32_t wnot(uint32_t a) { return ~a; }
+__host__ __device__ __forceinline__ unsigned long long wnot(unsigned long long a) { return ~a; }
+__host__ __device__ __forceinline__ u128 wnot(u128 a) { return {~a.lo, ~a.hi}; }
+
 __host__ __device__ __forceinline__ bool wzero(uint32_t a) { return a == 0; }
 __host__ __device__ __forceinline__ bool wzero(unsigned long long a) { return a == 0; }
 __host__ __device__ __forceinline__ bool wzero(u128 a) { return (a.lo | a.hi) == 0; }
@@ -56,6 +60,16 @@ __device__ __forceinline__ uint32_t wpiece(unsigned long long a, int k) { return
 __device__ __forceinline__ uint32_t wpiece(u128 a, int k) {
   unsigned long long h = (k < 2) ? a.lo : a.hi;
   return (uint32_t)(h >> (32 * (k & 1)));
+}
+
+// word from its 32-bit pieces (little-endian)
+template <typename T> __device__ __forceinline__ T wfrom_pieces(const uint32_t *p);
+template <> __device__ __forceinline__ uint32_t wfrom_pieces<uint32_t>(const uint32_t *p) { return p[0]; }
+template <> __device__ __forceinline__ unsigned long long wfrom_pieces<unsigned long long>(const uint32_t *p) {
+  return ((unsigned long long)p[1] << 32) | p[0];
+}
+template <> __device__ __forceinline__ u128 wfrom_pieces<u128>(const uint32_t *p) {
+  return {((unsigned long long)p[1] << 32) | p[0], ((unsigned long long)p[3] << 32) | p[2]};
 }
 
 // Bits [h * W/2, (h + 1) * W/2) of a word, h in {0, 1}, right-aligned.
@@ -97,6 +111,16 @@ __device__ __forceinline__ unsigned long long ldv(const unsigned long long *p) {
 __device__ __forceinline__ u128 ldv(const u128 *p) {
   const volatile unsigned long long *q = (const volatile unsigned long long *)p;
   return {q[0], q[1]};
+}
+
+// L2-coherent loads (ld.global.cg: skip L1) of words another CTA of this launch wrote
+// before a grid barrier.
+__device__ __forceinline__ uint32_t ldcg(const uint32_t *p) { return __ldcg(p); }
+__device__ __forceinline__ uint32_t ldcg_w(const uint32_t *p) { return __ldcg(p); }
+__device__ __forceinline__ unsigned long long ldcg_w(const unsigned long long *p) { return __ldcg(p); }
+__device__ __forceinline__ u128 ldcg_w(const u128 *p) {
+  ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2 *>(p));
+  return {v.x, v.y};
 }
 
 __device__ __forceinline__ uint32_t ld(const uint32_t *p) { return *p; }

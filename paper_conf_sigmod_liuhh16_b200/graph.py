@@ -198,8 +198,12 @@ class Graph:
     def run(self, sources, group_bits: int = 128, out="device", direction: str = "auto",
             schedule: str | None = None, bu_from: int = 2, alpha: float = 4.0, beta: float = 24.0,
             groups_in_flight: int = 0, stream=None, timing: bool = False, want_m: bool = True,
-            want_digest: bool = False, level_cap: int = 130):
+            want_digest: bool = False, level_cap: int = 130, split: str = "auto",
+            split_mod: int = 2, split_div: float = 64.0):
         """n concurrent BFS instances; returns (depths, RunStats).
+
+        split: "auto" | "off" | "force" -- per-instance direction inside a bottom-up level
+        (include/ibfs.h IBFS_SPLIT_*); never changes results.
 
         out: "device" (allocate a torch int8 [n, nv] CUDA tensor), "host" (numpy), None
         (no rows returned; they are still materialised on the device), or a caller buffer
@@ -240,6 +244,9 @@ class Graph:
                 stream = None
         opts.cuda_stream = getattr(stream, "cuda_stream", stream) or None
         opts.timing = 1 if timing else 0
+        opts.split = {"auto": 0, "off": 1, "force": 2}[split]
+        opts.split_mod = int(split_mod)
+        opts.split_div = float(split_div)
         st = _lib.Stats()
         m_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_m else None
         d_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_digest else None

@@ -61,6 +61,21 @@ def test_fig1_all_schedules(W, kind):
     np.testing.assert_array_equal(st.per_source_digest, ref.digest)
 
 
+@pytest.mark.parametrize("W", [32, 128])
+@pytest.mark.parametrize("kind", ["bu1", "bu2", "alt", "rand"])
+@pytest.mark.parametrize("mod", [1, 2, 3])
+def test_fig1_split_levels(W, kind, mod):
+    # per-instance split of BU levels (IBFS_SPLIT_FORCE): instances j % mod == 0 run
+    # top-down inside every BU level; results never change
+    fx = read_fig1()
+    el = ibfs_gen.from_pairs(fx["nv"], fx["edges"])
+    g = P.Graph.from_edgelist(el)
+    d, st = gpu_depths(g, fx["sources"], W, split="force", split_mod=mod, **run_kwargs(kind))
+    np.testing.assert_array_equal(d, fx["depths"])
+    ref = oracle.bfs(el, fx["sources"])
+    np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+
+
 def test_fig1_trace_frontiers():
     # SURVEY App. A trace (TD, TD, BU, ...): JFQ sizes 4, 6, then all 9 vertices in BU.
     fx = read_fig1()
@@ -88,10 +103,13 @@ def test_random_tiny_multigraphs_forced_schedules():
         src = rng.integers(0, nv, size=n).astype(np.uint32)  # duplicates allowed
         W = int(rng.choice([32, 64, 128]))
         kind = SCHEDULES[trial % len(SCHEDULES)]
+        split = ["auto", "off", "force"][trial % 3]
+        mod = int(rng.integers(1, 6))
         g = P.Graph.from_edgelist(el)
-        d, st = gpu_depths(g, src, W, groups_in_flight=int(rng.integers(0, 4)), **run_kwargs(kind, rng))
+        d, st = gpu_depths(g, src, W, groups_in_flight=int(rng.integers(0, 4)), split=split, split_mod=mod,
+                           **run_kwargs(kind, rng))
         ref = oracle.bfs(el, src)
-        np.testing.assert_array_equal(d, ref.depths, err_msg=f"trial {trial} W={W} {kind}")
+        np.testing.assert_array_equal(d, ref.depths, err_msg=f"trial {trial} W={W} {kind} split={split}/{mod}")
         np.testing.assert_array_equal(st.per_source_m, ref.m_s)
 
 
@@ -108,13 +126,14 @@ def _check_full(el, src, W, **kw):
 
 
 @pytest.mark.parametrize("kind", ["auto", "td", "bu2"])
-def test_config1_full(kind):
+@pytest.mark.parametrize("split", ["auto", "off", "force"])
+def test_config1_full(kind, split):
     cfg = ibfs_gen.CONFIGS["c1"]
     el = cfg.edges()
     src = cfg.sources(el)
     g = P.Graph.from_edgelist(el)
     perm = g.plan(src, cfg.group_bits)
-    _check_full(el, src[perm], cfg.group_bits, **run_kwargs(kind))
+    _check_full(el, src[perm], cfg.group_bits, split=split, split_mod=3, **run_kwargs(kind))
 
 
 @pytest.mark.parametrize("W", [32, 64, 128])
@@ -157,12 +176,14 @@ def test_config2_td_only_sd_counters_match_oracle():
     assert [x["new_pairs"] for x in st.per_level] == [x["new_pairs"] for x in lc]
 
 
-def test_config2_auto_level_counters_match_oracle():
+@pytest.mark.parametrize("split", ["auto", "off", "force"])
+def test_config2_auto_level_counters_match_oracle(split):
+    # a split BU level counts as bottom-up in Eq. 1 (reading #23 over all active instances)
     cfg = ibfs_gen.CONFIGS["c2"]
     el = cfg.edges()
     src = cfg.sources(el)
     g = P.Graph.from_edgelist(el)
-    d, st = gpu_depths(g, src, 128)
+    d, st = gpu_depths(g, src, 128, split=split, split_mod=2)
     ref = _oracle_c2(el, src)
     np.testing.assert_array_equal(d, ref.depths)
     sched = "".join("T" if x["td_groups"] else "B" for x in st.per_level)

@@ -29,14 +29,14 @@ done
 NCU_CFG=${NCU_CFG:-c5}
 if has launches; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none \
-    -k regex:'expand_kernel|commit_kernel|depth_kernel|init_|digest_kernel' \
+    -k regex:'level_kernel|expand_kernel|commit_kernel|depth_kernel|init_|digest_kernel' \
     --csv --log-file "$OUT/launches_$NCU_CFG.csv" \
     python bench.py --config $NCU_CFG --steps 2 --warmup 1 --no-e2e --no-cpu-baseline > "$OUT/launches_$NCU_CFG.log" 2>&1
   echo "launches rc=$?" >> "$OUT/launches_$NCU_CFG.log"
 fi
 if has full; then
   timeout 1200 ncu --set full --clock-control none --import-source on \
-    -k regex:'expand_kernel' -s ${NCU_SKIP:-6} -c ${NCU_COUNT:-3} -o "$OUT/expand_$NCU_CFG" \
+    -k regex:${NCU_KREGEX:-level_kernel} -s ${NCU_SKIP:-6} -c ${NCU_COUNT:-3} -o "$OUT/full_${NCU_KREGEX:-level_kernel}_$NCU_CFG" \
     python bench.py --config $NCU_CFG --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > "$OUT/full_$NCU_CFG.log" 2>&1
   echo "full rc=$?" >> "$OUT/full_$NCU_CFG.log"
 fi

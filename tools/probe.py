@@ -18,13 +18,15 @@ kw = {}
 for k, v in extra.items():
     kw[k] = float(v) if k in ("alpha", "beta") else (int(v) if v.isdigit() else v)
 iters = int(os.environ.get("PROBE_ITERS", 4))
-for it in range(iters):
-    ss = s[(it * G * 128) % len(s):][: G * 128]
+g0s = [int(x) for x in os.environ.get("PROBE_GROUPS", "").split(",") if x]
+for it in range(len(g0s) or iters):
+    g0 = g0s[it] if g0s else it * G
+    ss = s[(g0 * 128) % len(s):][: G * 128]
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     _, st = g.run(ss, 128, out=out[: len(ss)], timing=True, **kw)
     t1 = time.perf_counter()
-    print(f"{name} it{it}: wall {1e3*(t1-t0):.1f} ms traverse {st.traverse_ms:.1f} finalize {st.finalize_ms:.1f} "
+    print(f"{name} it{it} g0={g0}: wall {1e3*(t1-t0):.1f} ms traverse {st.traverse_ms:.1f} finalize {st.finalize_ms:.1f} "
           f"level {st.level_ms:.1f} (expand {st.expand_ms:.1f} commit {st.commit_ms:.1f}) depth {st.depth_ms:.1f} init {st.init_ms:.1f} "
           f"levels {st.max_levels} td {st.levels_td} bu {st.levels_bu} gteps {st.gteps:.0f} launches {st.n_launches}")
     for i, L in enumerate(st.per_level):

@@ -163,7 +163,12 @@ typedef struct {
   uint32_t split;             /* IBFS_SPLIT_* (default AUTO) */
   uint32_t split_mod;         /* IBFS_SPLIT_FORCE: instances j with j % split_mod == 0 */
   float split_div;            /* IBFS_SPLIT_AUTO ratio (default 64) */
-  uint32_t reserved[4];
+  /* k-hop mode (the reachability index of §8.7: "computes the first k
+     levels BFS for a large amount of selected vertices"; Table 1 uses k = 3).  max_depth
+     = k >= 1 stops every group after level k: vertices farther than k hops stay -1 and
+     m_s counts the vertices within k hops.  0 = unbounded (plain BFS, the default). */
+  uint32_t max_depth;
+  uint32_t reserved[3];
 } ibfs_run_opts;
 
 enum {

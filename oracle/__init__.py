@@ -59,6 +59,8 @@ def _load():
         lib.oracle_graph_export.argtypes = [P, P, P]
         lib.oracle_bfs.restype = ctypes.c_int
         lib.oracle_bfs.argtypes = [P, P, ctypes.c_uint64, P, P, P, P, P, ctypes.c_int]
+        lib.oracle_bfs_k.restype = ctypes.c_int
+        lib.oracle_bfs_k.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int32, P, P, P, P, P, ctypes.c_int]
         _lib = lib
     return _lib
 
@@ -118,8 +120,13 @@ class OracleGraph:
         off, _ = self.adjacency()
         return np.diff(off).astype(np.uint64)
 
-    def bfs(self, sources, want_depths: bool = True, threads: int | None = None) -> OracleResult:
-        """One textbook BFS per source.  depths: int8 [n][nv], row r <-> sources[r]."""
+    def bfs(self, sources, want_depths: bool = True, threads: int | None = None,
+            max_depth: int | None = None) -> OracleResult:
+        """One textbook BFS per source.  depths: int8 [n][nv], row r <-> sources[r].
+
+        max_depth = k caps every search at its first k levels -- the k-hop reachability
+        index of §8.7 ("computes the first k levels BFS"): vertices farther
+        than k hops are -1, and m_s / digest / reached count the vertices within k hops."""
         lib = _load()
         src = np.ascontiguousarray(np.asarray(sources, dtype=np.uint32))
         n = int(src.shape[0])
@@ -129,7 +136,10 @@ class OracleGraph:
             res.depths = np.empty((n, self.nv), dtype=np.int8)
             out_ptr = res.depths.ctypes.data
         t = threads or os.cpu_count() or 1
-        res.status = lib.oracle_bfs(self._h, src.ctypes.data if n else None, n, out_ptr,
+        k = -1 if max_depth is None else int(max_depth)
+        if max_depth is not None and k < 0:
+            raise ValueError("max_depth must be >= 0")
+        res.status = lib.oracle_bfs_k(self._h, src.ctypes.data if n else None, n, k, out_ptr,
                                     res.m_s.ctypes.data, res.digest.ctypes.data, res.ecc.ctypes.data,
                                     res.reached.ctypes.data, int(t))
         if res.status not in (0, ORACLE_E_RANGE):
@@ -137,8 +147,8 @@ class OracleGraph:
         return res
 
 
-def bfs(el, sources, want_depths=True, threads=None) -> OracleResult:
-    return OracleGraph.from_edges(el).bfs(sources, want_depths, threads)
+def bfs(el, sources, want_depths=True, threads=None, max_depth=None) -> OracleResult:
+    return OracleGraph.from_edges(el).bfs(sources, want_depths, threads, max_depth)
 
 
 from . import planner, stats, certify  # noqa: E402,F401

@@ -144,10 +144,14 @@ typedef struct {
   uint64_t next;      /* dynamic ticket */
   pthread_mutex_t lock;
   int status;
+  int32_t kmax;       /* -1 = unbounded */
 } bfs_job;
 
-/* One textbook BFS from s into dist (int32, -1 = unvisited).  Returns max depth. */
-static int32_t bfs_one(const oracle_graph *g, uint32_t s, int32_t *dist, uint32_t *queue,
+/* One textbook BFS from s into dist (int32, -1 = unvisited).  Returns max depth.
+ * kmax >= 0 caps the search at the first kmax levels (the k-hop reachability index of
+ * §8.7: "computes the first k levels BFS"): a vertex at depth kmax is
+ * recorded but not expanded, so every vertex farther than kmax hops stays -1. */
+static int32_t bfs_one(const oracle_graph *g, uint32_t s, int32_t kmax, int32_t *dist, uint32_t *queue,
                        uint64_t *m_out, uint64_t *dig_out, uint64_t *reached_out) {
   uint64_t head = 0, tail = 0;
   for (uint64_t x = 0; x < g->nv; ++x) dist[x] = -1;
@@ -161,6 +165,7 @@ static int32_t bfs_one(const oracle_graph *g, uint32_t s, int32_t *dist, uint32_
     if (dx > ecc) ecc = dx;
     m += g->off[x + 1] - g->off[x];
     dig += splitmix64(((uint64_t)x << 8) | (uint64_t)(dx + 1));
+    if (kmax >= 0 && dx >= kmax) continue;
     for (uint64_t k = g->off[x]; k < g->off[x + 1]; ++k) {
       uint32_t w = g->adj[k];
       if (dist[w] == -1) {
@@ -193,7 +198,7 @@ static void *bfs_worker(void *arg) {
     pthread_mutex_unlock(&j->lock);
     if (r >= j->n) break;
     uint64_t m, dig, reached;
-    int32_t ecc = bfs_one(g, j->sources[r], dist, queue, &m, &dig, &reached);
+    int32_t ecc = bfs_one(g, j->sources[r], j->kmax, dist, queue, &m, &dig, &reached);
     if (ecc > 127) {
       pthread_mutex_lock(&j->lock);
       j->status = ORACLE_E_RANGE;
@@ -213,9 +218,10 @@ static void *bfs_worker(void *arg) {
   return NULL;
 }
 
-/* Run n textbook BFSes (one per source) on `threads` worker threads. */
-int oracle_bfs(const oracle_graph *g, const uint32_t *sources, uint64_t n, int8_t *out,
-               uint64_t *m_s, uint64_t *digest, int32_t *ecc, uint64_t *reached, int threads) {
+/* Run n textbook BFSes (one per source) on `threads` worker threads, each capped at
+ * max_depth levels (max_depth < 0: unbounded). */
+int oracle_bfs_k(const oracle_graph *g, const uint32_t *sources, uint64_t n, int32_t max_depth, int8_t *out,
+                 uint64_t *m_s, uint64_t *digest, int32_t *ecc, uint64_t *reached, int threads) {
   if (!g || (n && !sources)) return ORACLE_E_INVALID;
   for (uint64_t r = 0; r < n; ++r)
     if (sources[r] >= g->nv) return ORACLE_E_INVALID;
@@ -226,6 +232,7 @@ int oracle_bfs(const oracle_graph *g, const uint32_t *sources, uint64_t n, int8_
   job.g = g; job.sources = sources; job.n = n; job.out = out; job.m_s = m_s;
   job.digest = digest; job.ecc = ecc; job.reached = reached; job.next = 0;
   job.status = ORACLE_OK;
+  job.kmax = max_depth < 0 ? -1 : max_depth;
   pthread_mutex_init(&job.lock, NULL);
   pthread_t *tid = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)threads);
   if (!tid) return ORACLE_E_NOMEM;
@@ -235,4 +242,9 @@ int oracle_bfs(const oracle_graph *g, const uint32_t *sources, uint64_t n, int8_
   free(tid);
   pthread_mutex_destroy(&job.lock);
   return job.status;
+}
+
+int oracle_bfs(const oracle_graph *g, const uint32_t *sources, uint64_t n, int8_t *out,
+               uint64_t *m_s, uint64_t *digest, int32_t *ecc, uint64_t *reached, int threads) {
+  return oracle_bfs_k(g, sources, n, -1, out, m_s, digest, ecc, reached, threads);
 }

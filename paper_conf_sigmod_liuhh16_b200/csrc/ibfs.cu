@@ -933,6 +933,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.pol.split = o.split;
   a.pol.split_mod = std::max<uint32_t>(1, o.split_mod);
   a.pol.split_div = o.split_div;
+  a.pol.max_depth = o.max_depth;
   a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
   for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
   uint32_t first_dir = 0;

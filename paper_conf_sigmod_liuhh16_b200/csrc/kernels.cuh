@@ -96,6 +96,7 @@ struct Policy {
   uint32_t sched_len;
   uint32_t split, split_mod;  // IBFS_SPLIT_*
   float split_div;
+  uint32_t max_depth;  // k-hop cap (0 = unbounded)
   uint8_t sched[MAXL];  // 0 TD / 1 BU for level l at index l-1
 };
 
@@ -1079,7 +1080,7 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->arrive = 0;
     c->last_level = (uint32_t)lc;
     for (int k = 0; k < NQ; ++k) c->qlen[(lc + 1) & 1][k] = 0;  // target of commit lc+1
-    if (wzero(act)) {
+    if (wzero(act) || (a.pol.max_depth != 0 && (uint32_t)lc >= a.pol.max_depth)) {
       c->done = 1;
       __threadfence();
       atomicAdd(a.batch_done, 1u);

@@ -199,8 +199,11 @@ class Graph:
             schedule: str | None = None, bu_from: int = 2, alpha: float = 4.0, beta: float = 24.0,
             groups_in_flight: int = 0, stream=None, timing: bool = False, want_m: bool = True,
             want_digest: bool = False, level_cap: int = 130, split: str = "auto",
-            split_mod: int = 2, split_div: float = 64.0):
+            split_mod: int = 2, split_div: float = 64.0, max_depth: int | None = None):
         """n concurrent BFS instances; returns (depths, RunStats).
+
+        max_depth = k >= 1: k-hop mode, the first k levels only (the reachability index of
+        §8.7); vertices farther than k hops are -1.  None = plain BFS.
 
         split: "auto" | "off" | "force" -- per-instance direction inside a bottom-up level
         (include/ibfs.h IBFS_SPLIT_*); never changes results.
@@ -247,6 +250,10 @@ class Graph:
         opts.split = {"auto": 0, "off": 1, "force": 2}[split]
         opts.split_mod = int(split_mod)
         opts.split_div = float(split_div)
+        if max_depth is not None:
+            if int(max_depth) < 1:
+                raise ValueError("max_depth must be >= 1 (None = unbounded)")
+            opts.max_depth = int(max_depth)
         st = _lib.Stats()
         m_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_m else None
         d_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_digest else None

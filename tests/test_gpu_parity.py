@@ -335,3 +335,49 @@ def test_torch_allocator_hook():
     finally:
         P.use_torch_allocator(False)
     np.testing.assert_array_equal(d, oracle.bfs(el, s).depths)
+
+
+# ------------------------------------------------- k-hop reachability index (NEXT #2)
+# §8.7: "computes the first k levels BFS for a large amount of selected
+# vertices"; Table 1 builds the 3-hop index.  Oracle: the same textbook BFS capped at k.
+@pytest.mark.parametrize("k", [1, 2, 3, 5])
+@pytest.mark.parametrize("kind", ["auto", "td", "bu1", "rand"])
+def test_khop_fig1_and_tiny(k, kind):
+    rng = np.random.default_rng(100 + k)
+    for trial in range(20):
+        nv = int(rng.integers(1, 50))
+        m = int(rng.integers(0, 3 * nv + 1))
+        pairs = [(int(rng.integers(nv)), int(rng.integers(nv))) for _ in range(m)]
+        el = ibfs_gen.from_pairs(nv, pairs if pairs else np.zeros((0, 2)))
+        n = int(rng.integers(1, 150))
+        src = rng.integers(0, nv, size=n).astype(np.uint32)
+        W = int(rng.choice([32, 64, 128]))
+        g = P.Graph.from_edgelist(el)
+        d, st = gpu_depths(g, src, W, max_depth=k, want_digest=True, **run_kwargs(kind, rng))
+        ref = oracle.bfs(el, src, max_depth=k)
+        np.testing.assert_array_equal(d, ref.depths, err_msg=f"trial {trial} k={k} {kind} W={W}")
+        np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+        np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+        assert st.max_levels <= k
+
+
+@pytest.mark.parametrize("k", [1, 2, 3])
+def test_khop_config2_full(k):
+    cfg = ibfs_gen.CONFIGS["c2"]
+    el = cfg.edges()
+    src = cfg.sources(el)
+    g = P.Graph.from_edgelist(el)
+    s = src[g.plan(src, 128)]
+    d, st = gpu_depths(g, s, 128, max_depth=k, want_digest=True)
+    ref = oracle.bfs(el, s, max_depth=k)
+    np.testing.assert_array_equal(d, ref.depths)
+    np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+    np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+    full = _oracle_c2(el, s)
+    np.testing.assert_array_equal(d, np.where(full.depths <= k, full.depths, -1))
+
+
+def test_khop_invalid():
+    g = P.Graph.from_edgelist(ibfs_gen.from_pairs(4, [(0, 1)]))
+    with pytest.raises(ValueError):
+        g.run(np.array([0], dtype=np.uint32), 32, max_depth=0)

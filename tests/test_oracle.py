@@ -215,3 +215,51 @@ def test_thread_count_invariance():
     b = g.bfs(srcs, threads=7)
     np.testing.assert_array_equal(a.depths, b.depths)
     np.testing.assert_array_equal(a.digest, b.digest)
+
+
+# ---- k-hop reachability index (§8.7: "the first k levels BFS") ----------
+
+@pytest.mark.parametrize("directed", [False, True])
+def test_khop_floyd_warshall_random_tiny(directed):
+    """depth capped at k == the brute-force distance where it is <= k, else -1; m_s and
+    reached count exactly the vertices within k hops (degrees from the raw tuples)."""
+    rng = np.random.default_rng(777 + directed)
+    for trial in range(300):
+        nv = int(rng.integers(1, 31))
+        m = int(rng.integers(0, 2 * nv + 1))
+        pairs = random_multigraph(rng, nv, m)
+        fw = floyd_warshall(nv, pairs, directed)
+        deg = np.zeros(nv, dtype=np.int64)
+        for u, v in pairs:
+            deg[u] += 1
+            if not directed:
+                deg[v] += 1
+        k = int(rng.integers(0, 5))
+        el = ibfs_gen.from_pairs(nv, pairs if pairs else np.zeros((0, 2)), directed)
+        res = oracle.OracleGraph.from_edges(el).bfs(np.arange(nv, dtype=np.uint32), max_depth=k)
+        exp = np.where((fw >= 0) & (fw <= k), fw, -1)
+        np.testing.assert_array_equal(res.depths.astype(np.int64), exp, err_msg=f"trial {trial} k={k}")
+        within = exp >= 0
+        np.testing.assert_array_equal(res.reached.astype(np.int64), within.sum(axis=1))
+        np.testing.assert_array_equal(res.m_s.astype(np.int64), (within * deg[None, :]).sum(axis=1))
+
+
+def test_khop_closed_forms():
+    """Path graph: d = |i - j| where <= k; k = 0 keeps only the source; k >= the diameter
+    is the plain BFS."""
+    n = 40
+    pairs = [(i, i + 1) for i in range(n - 1)]
+    el = ibfs_gen.from_pairs(n, pairs, False)
+    g = oracle.OracleGraph.from_edges(el)
+    ii, jj = np.meshgrid(np.arange(n), np.arange(n), indexing="ij")
+    dd = np.abs(ii - jj)
+    for k in (0, 1, 3, 7):
+        r = g.bfs(np.arange(n, dtype=np.uint32), max_depth=k)
+        np.testing.assert_array_equal(r.depths, np.where(dd <= k, dd, -1))
+        assert (r.ecc == np.minimum(k, np.maximum(np.arange(n), n - 1 - np.arange(n)))).all()
+    full = g.bfs(np.arange(n, dtype=np.uint32))
+    capped = g.bfs(np.arange(n, dtype=np.uint32), max_depth=n - 1)
+    np.testing.assert_array_equal(full.depths, capped.depths)
+    np.testing.assert_array_equal(full.digest, capped.digest)
+    with pytest.raises(ValueError):
+        g.bfs(np.arange(2, dtype=np.uint32), max_depth=-1)

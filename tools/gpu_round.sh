@@ -29,7 +29,7 @@ done
 NCU_CFG=${NCU_CFG:-c5}
 if has launches; then
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none \
-    -k regex:'level_kernel|expand_kernel|commit_kernel|depth_kernel|init_|digest_kernel' \
+    -k regex:'level_kernel|depth_kernel|init_|ms_kernel|iso_fix|digest_kernel' \
     --csv --log-file "$OUT/launches_$NCU_CFG.csv" \
     python bench.py --config $NCU_CFG --steps 2 --warmup 1 --no-e2e --no-cpu-baseline > "$OUT/launches_$NCU_CFG.log" 2>&1
   echo "launches rc=$?" >> "$OUT/launches_$NCU_CFG.log"

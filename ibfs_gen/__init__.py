@@ -122,9 +122,12 @@ class Config:
     group_bits: int
     graph_seed: int = 1
     source_seed: int = 2
+    directed: bool = False  # tuple (u, v) = the edge u->v only
 
     def edges(self, threads=None) -> EdgeList:
-        return rmat(self.scale, self.ef, self.abc, self.graph_seed, True, threads)
+        el = rmat(self.scale, self.ef, self.abc, self.graph_seed, True, threads)
+        el.directed = self.directed
+        return el
 
     def sources(self, el: EdgeList) -> np.ndarray:
         if self.n_sources == 0:
@@ -138,4 +141,6 @@ CONFIGS = {
     "c3": Config("c3: R-MAT s24 ef32, i=1024", RMAT, 24, 32, 1024, 128),
     "c4": Config("c4: Kronecker s18 ef16, APSP i=|V|", KRONECKER, 18, 16, 0, 128),
     "c5": Config("c5: Kronecker s26 ef16, i=4096", KRONECKER, 26, 16, 4096, 128),
+    # directed parity case (NEXT #1): config 2's tuples read as directed edges u->v
+    "d2": Config("d2: directed Kronecker s20 ef16, i=128", KRONECKER, 20, 16, 128, 128, directed=True),
 }

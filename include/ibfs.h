@@ -34,7 +34,7 @@ typedef enum {
   IBFS_E_NOMEM = -2,       /* device or host allocation failed */
   IBFS_E_CUDA = -3,        /* CUDA runtime error, or no usable device */
   IBFS_E_RANGE = -4,       /* some depth > 127 does not fit the int8 output */
-  IBFS_E_UNSUPPORTED = -5  /* valid request this build does not implement (directed BU) */
+  IBFS_E_UNSUPPORTED = -5  /* valid request this build does not implement (degree >= 2^32) */
 } ibfs_status;
 
 typedef struct ibfs_graph ibfs_graph; /* opaque; owned by the library */
@@ -52,9 +52,12 @@ const char *ibfs_last_error(void);
  * ibfs_load_csr: copy a CSR into device memory owned by the library on `device`.
  *   offsets[nv + 1] (u64): offsets[0] = 0, non-decreasing, offsets[nv] = ne.
  *   adj[ne] (u32): every id < nv.  Undirected graphs pass the symmetrized CSR and
- *   rev_offsets = rev_adj = NULL (bottom-up reads the same rows).  Directed graphs need
- *   the reverse (in-edge) CSR for bottom-up: not implemented in this build ->
- *   IBFS_E_UNSUPPORTED when rev_* are non-NULL.
+ *   rev_offsets = rev_adj = NULL (bottom-up reads the same rows).  Directed graphs pass
+ *   the out-edge CSR in offsets/adj (top-down expands it) and its transpose, the in-edge
+ *   CSR, in rev_offsets[nv + 1] / rev_adj[ne] ("for directed graphs, we also store the
+ *   reverse edges"; bottom-up reads a vertex's parents from it).  The transpose
+ *   is checked by degree sequences (every vertex's occurrences in adj == its rev row
+ *   length and vice versa) -> IBFS_E_INVALID; it is not otherwise verified.
  *   Inputs may be host or device pointers; they are neither retained nor modified.
  *   nv >= 1, ne < 2^40.  On success *out_graph owns all device state; release with
  *   ibfs_free.
@@ -67,11 +70,14 @@ int ibfs_load_csr(int device, uint32_t nv, uint64_t ne, const uint64_t *offsets,
  *   e < n_tuples (host or device pointers).  Undirected (directed = 0): tuple (u, v)
  *   yields entries u->v and v->u; duplicates and self-loops are kept (a self-loop tuple
  *   gives two entries), and each row keeps tuple order (stable) -- P:L887.
- *   directed != 0 -> IBFS_E_UNSUPPORTED in this build. */
+ *   Directed (directed != 0): tuple (u, v) is the edge u->v only; the library builds
+ *   the out-edge rows (top-down) and the in-edge rows (bottom-up), both in tuple order. */
 int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const uint32_t *u,
                     const uint32_t *v, int directed, ibfs_graph **out_graph);
 
-/* Row order of the device adjacency (never changes any result):
+/* Row order of the device adjacency (never changes any result).  Applies
+ * to the rows bottom-up scans: the CSR of an undirected graph, the in-edge rows of a
+ * directed one (keyed by the parent's in-degree).
  *   IBFS_ROWS_KEEP      keep the loaded order (tuple order for ibfs_load_edges).
  *   IBFS_ROWS_HUB_FIRST stable-sort every row by neighbour outdegree, descending, so
  *                       bottom-up inspection (Alg. 1) meets the vertices most
@@ -83,7 +89,8 @@ int ibfs_graph_sort_rows(ibfs_graph *g, int order);
 int ibfs_graph_info(const ibfs_graph *g, uint32_t *nv, uint64_t *ne, uint32_t *max_degree,
                     int *device);
 
-/* Copy the device CSR back to caller-allocated HOST arrays offsets[nv+1], adj[ne]. */
+/* Copy the device CSR (the out-edge rows of a directed graph) back to caller-allocated
+ * HOST arrays offsets[nv+1], adj[ne]. */
 int ibfs_graph_export_csr(const ibfs_graph *g, uint64_t *offsets, uint32_t *adj);
 
 /* Release everything g owns.  NULL-safe. */

@@ -183,6 +183,20 @@ struct ibfs_graph {
   uint32_t *d_hub_chunk0 = nullptr;  // [n_hubs + 1] first chunk of each hub
   uint32_t n_hubs = 0;
   std::vector<uint64_t> h_off;      // host copy of d_off (tiling, planner)
+  // Directed graphs ("store the reverse edges" for bottom-up): the in-edge CSR in
+  // the same compacted space (a vertex is kept if it has an out- or an in-edge), with its
+  // own degrees and hub chunks.  Undirected: directed = false and none of these is
+  // allocated (the kernels read the out-edge arrays for both directions).
+  bool directed = false;
+  unsigned long long *d_roff = nullptr;
+  uint32_t *d_radj = nullptr;
+  uint32_t *d_rdeg = nullptr;
+  HubChunk *d_rchunks = nullptr;
+  uint32_t n_rchunks = 0;
+  uint32_t *d_rhub_vtx = nullptr;
+  uint32_t *d_rhub_chunk0 = nullptr;
+  uint32_t n_rhubs = 0;
+  std::vector<uint64_t> h_roff;
   std::vector<uint32_t> h_tbase, h_nzbits;
   int num_sms = 148;
   int level_blocks_per_sm[3] = {1, 1, 1};  // co-resident level_kernel CTAs per SM (W = 32, 64, 128)
@@ -202,6 +216,12 @@ void graph_release(ibfs_graph *g) {
   cudaFree(g->d_hub_chunk0);
   cudaFree(g->d_tbase);
   cudaFree(g->d_nzbits);
+  cudaFree(g->d_roff);
+  cudaFree(g->d_radj);
+  cudaFree(g->d_rdeg);
+  cudaFree(g->d_rchunks);
+  cudaFree(g->d_rhub_vtx);
+  cudaFree(g->d_rhub_chunk0);
   if (prev >= 0) cudaSetDevice(prev);
   cudaGetLastError();
   delete g;
@@ -236,10 +256,12 @@ __global__ void max_id_kernel(const uint32_t *adj, unsigned long long ne, uint32
 }
 
 // ---- compaction ----
-__global__ void nzbits_kernel(const unsigned long long *off, uint32_t nv, uint32_t *nzbits) {
+// a vertex is kept when it has an out-edge or (directed, roff != NULL) an in-edge
+__global__ void nzbits_kernel(const unsigned long long *off, const unsigned long long *roff, uint32_t nv,
+                              uint32_t *nzbits) {
   const size_t nvr = ((size_t)nv + 31) & ~(size_t)31;
   for (size_t v = (size_t)blockIdx.x * blockDim.x + threadIdx.x; v < nvr; v += (size_t)gridDim.x * blockDim.x) {
-    const bool nz = v < nv && off[v + 1] > off[v];
+    const bool nz = v < nv && (off[v + 1] > off[v] || (roff && roff[v + 1] > roff[v]));
     const uint32_t b = __ballot_sync(FULL, nz);
     if ((threadIdx.x & 31) == 0) nzbits[v >> 5] = b;
   }
@@ -274,8 +296,9 @@ __global__ void remap_adj_kernel(uint32_t *adj, unsigned long long ne, const uin
 }
 
 // d_off_orig [nv + 1] (caller ids, consumed and freed) and g->d_adj (caller ids, remapped in
-// place) -> compacted g->d_off, g->d_adj, g->d_tbase, g->d_nzbits, host copies.
-void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig) {
+// place) -> compacted g->d_off, g->d_adj, g->d_tbase, g->d_nzbits, host copies; for a
+// directed graph the same for d_roff_orig / g->d_radj -> g->d_roff, g->d_radj.
+void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig, unsigned long long *d_roff_orig = nullptr) {
   const uint32_t nv = g->nv;
   const uint32_t nwords = (nv + 31) / 32, ntiles = (nv + 127) / 128;
   // padded to whole 128-vertex tiles (+1) so a tile's 4 words load as one uint4
@@ -288,7 +311,7 @@ void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig) {
   try {
     CK(cudaMalloc(&cnt, ((size_t)ntiles + 1) * 4));
     CK(cudaMemset(cnt, 0, ((size_t)ntiles + 1) * 4));
-    nzbits_kernel<<<2048, 256>>>(d_off_orig, nv, g->d_nzbits);
+    nzbits_kernel<<<2048, 256>>>(d_off_orig, d_roff_orig, nv, g->d_nzbits);
     tilecount_kernel<<<(ntiles + 255) / 256, 256>>>(g->d_nzbits, nwords, ntiles, cnt);
     CK(cudaGetLastError());
     size_t tb = 0;
@@ -311,6 +334,7 @@ void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig) {
     cudaFree(cnt);
     cudaFree(tmp);
     cudaFree(d_off_orig);
+    cudaFree(d_roff_orig);
     throw;
   }
   cudaFree(cnt);
@@ -318,6 +342,23 @@ void compact_graph(ibfs_graph *g, unsigned long long *d_off_orig) {
   cudaFree(d_off_orig);
   g->h_off.resize((size_t)g->nva + 1);
   CK(cudaMemcpy(g->h_off.data(), g->d_off, ((size_t)g->nva + 1) * 8, cudaMemcpyDeviceToHost));
+  if (d_roff_orig) {
+    try {
+      CK(cudaMalloc(&g->d_roff, ((size_t)g->nva + 1) * sizeof(unsigned long long)));
+      const unsigned long long ne = g->ne;
+      CK(cudaMemcpy(g->d_roff + g->nva, &ne, sizeof(ne), cudaMemcpyHostToDevice));
+      compact_rows_kernel<<<2048, 256>>>(d_roff_orig, g->nv, g->d_tbase, g->d_nzbits, g->d_roff);
+      if (g->ne) remap_adj_kernel<<<4096, 256>>>(g->d_radj, g->ne, g->d_tbase, g->d_nzbits);
+      CK(cudaGetLastError());
+      CK(cudaDeviceSynchronize());
+    } catch (...) {
+      cudaFree(d_roff_orig);
+      throw;
+    }
+    cudaFree(d_roff_orig);
+    g->h_roff.resize((size_t)g->nva + 1);
+    CK(cudaMemcpy(g->h_roff.data(), g->d_roff, ((size_t)g->nva + 1) * 8, cudaMemcpyDeviceToHost));
+  }
 }
 
 // Host twin of compact_id for a caller id; NO_VERTEX if the vertex is isolated.
@@ -332,35 +373,36 @@ uint32_t host_compact_id(const ibfs_graph *g, uint32_t v) {
 
 // Static hub decomposition: the rows of vertices with degree > HUB_T are
 // cut into chunks of CHUNK edges, each a work item a whole CTA sweeps.
-void build_decomposition(ibfs_graph *g) {
+void build_decomposition(const std::vector<uint64_t> &h_off, uint32_t nva, HubChunk **d_chunks,
+                         uint32_t *n_chunks, uint32_t **d_hub_vtx, uint32_t **d_hub_chunk0, uint32_t *n_hubs) {
   std::vector<HubChunk> chunks;
   std::vector<uint32_t> hubs, chunk0;
-  for (uint32_t v = 0; v < g->nva; ++v) {
-    const uint64_t d = g->h_off[v + 1] - g->h_off[v];
+  for (uint32_t v = 0; v < nva; ++v) {
+    const uint64_t d = h_off[v + 1] - h_off[v];
     if (d <= (uint64_t)HUB_T) continue;
     hubs.push_back(v);
     chunk0.push_back((uint32_t)chunks.size());
     uint32_t first = 1;
-    for (uint64_t e = g->h_off[v]; e < g->h_off[v + 1]; e += CHUNK) {
+    for (uint64_t e = h_off[v]; e < h_off[v + 1]; e += CHUNK) {
       HubChunk c;
       c.e0 = e;
-      c.e1 = std::min<uint64_t>(e + CHUNK, g->h_off[v + 1]);
+      c.e1 = std::min<uint64_t>(e + CHUNK, h_off[v + 1]);
       c.v = v;
       c.first = first;
       first = 0;
       chunks.push_back(c);
     }
   }
-  g->n_chunks = (uint32_t)chunks.size();
-  chunk0.push_back(g->n_chunks);
-  g->n_hubs = (uint32_t)hubs.size();
-  CK(cudaMalloc(&g->d_chunks, std::max<size_t>(chunks.size(), 1) * sizeof(HubChunk)));
+  *n_chunks = (uint32_t)chunks.size();
+  chunk0.push_back(*n_chunks);
+  *n_hubs = (uint32_t)hubs.size();
+  CK(cudaMalloc(d_chunks, std::max<size_t>(chunks.size(), 1) * sizeof(HubChunk)));
   if (!chunks.empty())
-    CK(cudaMemcpy(g->d_chunks, chunks.data(), chunks.size() * sizeof(HubChunk), cudaMemcpyHostToDevice));
-  CK(cudaMalloc(&g->d_hub_vtx, std::max<size_t>(hubs.size(), 1) * 4));
-  CK(cudaMalloc(&g->d_hub_chunk0, chunk0.size() * 4));
-  if (!hubs.empty()) CK(cudaMemcpy(g->d_hub_vtx, hubs.data(), hubs.size() * 4, cudaMemcpyHostToDevice));
-  CK(cudaMemcpy(g->d_hub_chunk0, chunk0.data(), chunk0.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(*d_chunks, chunks.data(), chunks.size() * sizeof(HubChunk), cudaMemcpyHostToDevice));
+  CK(cudaMalloc(d_hub_vtx, std::max<size_t>(hubs.size(), 1) * 4));
+  CK(cudaMalloc(d_hub_chunk0, chunk0.size() * 4));
+  if (!hubs.empty()) CK(cudaMemcpy(*d_hub_vtx, hubs.data(), hubs.size() * 4, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(*d_hub_chunk0, chunk0.data(), chunk0.size() * 4, cudaMemcpyHostToDevice));
 }
 
 // Degrees, max degree, hub chunks; compacted offsets must be in g->d_off and g->h_off.
@@ -379,7 +421,20 @@ void finish_graph(ibfs_graph *g) {
       fail(IBFS_E_UNSUPPORTED, "vertex degree >= 2^32");
   g->max_deg = (uint32_t)h[0];
   g->nv_active = h[1];
-  build_decomposition(g);
+  build_decomposition(g->h_off, g->nva, &g->d_chunks, &g->n_chunks, &g->d_hub_vtx, &g->d_hub_chunk0, &g->n_hubs);
+  if (g->directed) {
+    CK(cudaMalloc(&g->d_rdeg, std::max<size_t>(g->nva, 1) * sizeof(uint32_t)));
+    CK(cudaMalloc(&d_stats, 2 * sizeof(unsigned long long)));
+    CK(cudaMemset(d_stats, 0, 2 * sizeof(unsigned long long)));
+    degree_kernel<<<1024, 256>>>(g->d_roff, g->nva, g->d_rdeg, d_stats);
+    CK(cudaGetLastError());
+    CK(cudaMemcpy(h, d_stats, sizeof(h), cudaMemcpyDeviceToHost));
+    cudaFree(d_stats);
+    for (uint32_t v = 0; v < g->nva; ++v)
+      if (g->h_roff[v + 1] - g->h_roff[v] > 0xffffffffull) fail(IBFS_E_UNSUPPORTED, "vertex in-degree >= 2^32");
+    build_decomposition(g->h_roff, g->nva, &g->d_rchunks, &g->n_rchunks, &g->d_rhub_vtx, &g->d_rhub_chunk0,
+                        &g->n_rhubs);
+  }
   int dev = g->device;
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev));
   CK(cudaFuncSetAttribute(level_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -405,24 +460,50 @@ void finish_graph(ibfs_graph *g) {
   set_pool_threshold(dev);
 }
 
-__global__ void explode_kernel(const uint32_t *u, const uint32_t *v, unsigned long long m,
-                               uint32_t *keys, uint32_t *vals, unsigned long long *deg, uint32_t nv,
-                               uint32_t *bad) {
+// undirected tuple (a, b) -> CSR entries a->b and b->a
+__global__ void explode_kernel(const uint32_t *u, const uint32_t *v, unsigned long long m, uint32_t *keys,
+                               uint32_t *vals) {
   for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m;
        e += (unsigned long long)gridDim.x * blockDim.x) {
-    uint32_t a = u[e], b = v[e];
-    if (a >= nv || b >= nv) {
-      *bad = 1;
-      a = 0;
-      b = 0;
-    }
+    const uint32_t a = u[e], b = v[e];
     keys[2 * e] = a;
     vals[2 * e] = b;
     keys[2 * e + 1] = b;
     vals[2 * e + 1] = a;
-    atomicAdd(deg + a, 1ull);
-    atomicAdd(deg + b, 1ull);
   }
+}
+
+__global__ void check_ids_kernel(const uint32_t *u, const uint32_t *v, unsigned long long m, uint32_t nv,
+                                 uint32_t *bad) {
+  for (unsigned long long e = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; e < m;
+       e += (unsigned long long)gridDim.x * blockDim.x)
+    if (u[e] >= nv || v[e] >= nv) *bad = 1;
+}
+
+__global__ void count_ids_kernel(const uint32_t *adj, unsigned long long ne, unsigned long long *cnt) {
+  for (unsigned long long i = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x; i < ne;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    atomicAdd(cnt + adj[i], 1ull);
+}
+
+// occurrences of every id in adj[ne] == the row lengths of the other CSR side (h_off)
+bool degrees_match(const uint32_t *d_adj, uint64_t ne, const std::vector<uint64_t> &h_off, uint32_t nv) {
+  unsigned long long *cnt = nullptr;
+  CK(cudaMalloc(&cnt, (size_t)nv * 8));
+  std::vector<unsigned long long> h(nv);
+  try {
+    CK(cudaMemset(cnt, 0, (size_t)nv * 8));
+    count_ids_kernel<<<4096, 256>>>(d_adj, ne, cnt);
+    CK(cudaGetLastError());
+    CK(cudaMemcpy(h.data(), cnt, (size_t)nv * 8, cudaMemcpyDeviceToHost));
+  } catch (...) {
+    cudaFree(cnt);
+    throw;
+  }
+  cudaFree(cnt);
+  for (uint32_t v = 0; v < nv; ++v)
+    if (h[v] != h_off[v + 1] - h_off[v]) return false;
+  return true;
 }
 
 }  // namespace
@@ -440,43 +521,55 @@ extern "C" int ibfs_load_csr(int device, uint32_t nv, uint64_t ne, const uint64_
     if (nv == 0) fail(IBFS_E_INVALID, "nv must be >= 1");
     if (!offsets || (ne > 0 && !adj)) fail(IBFS_E_INVALID, "offsets/adj is NULL");
     if (ne >= (1ull << 40)) fail(IBFS_E_INVALID, "ne too large");
-    if (rev_offsets || rev_adj)
-      fail(IBFS_E_UNSUPPORTED, "directed graphs (reverse CSR) are not implemented in this build");
+    const bool directed = rev_offsets != nullptr;
+    if (directed != (rev_adj != nullptr) && ne > 0) fail(IBFS_E_INVALID, "rev_offsets and rev_adj must both be set");
     DeviceScope ds(device);
     ibfs_graph *g = new ibfs_graph();
-    try {
-      g->device = device;
-      g->nv = nv;
-      g->ne = ne;
-      g->h_off.resize((size_t)nv + 1);
-      CK(cudaMemcpy(g->h_off.data(), offsets, ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyDefault));
-      if (g->h_off[0] != 0 || g->h_off[nv] != ne) fail(IBFS_E_INVALID, "offsets[0] != 0 or offsets[nv] != ne");
+    unsigned long long *d_off_orig = nullptr, *d_roff_orig = nullptr;
+    // one CSR side: validate the offsets on the host, copy both arrays, check the ids
+    auto load_side = [&](const uint64_t *o, const uint32_t *ad, std::vector<uint64_t> &h, unsigned long long **d_o,
+                         uint32_t **d_a) {
+      h.resize((size_t)nv + 1);
+      CK(cudaMemcpy(h.data(), o, ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyDefault));
+      if (h[0] != 0 || h[nv] != ne) fail(IBFS_E_INVALID, "offsets[0] != 0 or offsets[nv] != ne");
       for (uint32_t v = 0; v < nv; ++v)
-        if (g->h_off[v + 1] < g->h_off[v]) fail(IBFS_E_INVALID, "offsets not non-decreasing");
-      unsigned long long *d_off_orig = nullptr;
-      CK(cudaMalloc(&d_off_orig, ((size_t)nv + 1) * sizeof(unsigned long long)));
-      {
-        cudaError_t e = cudaMemcpy(d_off_orig, g->h_off.data(), ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice);
-        if (e != cudaSuccess) { cudaFree(d_off_orig); CK(e); }
-      }
-      g->d_off = d_off_orig;  // released by graph_release if a later step fails
-      CK(cudaMalloc(&g->d_adj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
-      if (ne) CK(cudaMemcpy(g->d_adj, adj, ne * sizeof(uint32_t), cudaMemcpyDefault));
+        if (h[v + 1] < h[v]) fail(IBFS_E_INVALID, "offsets not non-decreasing");
+      CK(cudaMalloc(d_o, ((size_t)nv + 1) * sizeof(unsigned long long)));
+      CK(cudaMemcpy(*d_o, h.data(), ((size_t)nv + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
+      CK(cudaMalloc(d_a, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
       if (ne) {
+        CK(cudaMemcpy(*d_a, ad, ne * sizeof(uint32_t), cudaMemcpyDefault));
         uint32_t *d_mx = nullptr;
         CK(cudaMalloc(&d_mx, sizeof(uint32_t)));
         CK(cudaMemset(d_mx, 0, sizeof(uint32_t)));
-        max_id_kernel<<<1024, 256>>>(g->d_adj, ne, d_mx);
+        max_id_kernel<<<1024, 256>>>(*d_a, ne, d_mx);
         CK(cudaGetLastError());
         uint32_t mx = 0;
         CK(cudaMemcpy(&mx, d_mx, sizeof(uint32_t), cudaMemcpyDeviceToHost));
         cudaFree(d_mx);
         if (mx >= nv) fail(IBFS_E_INVALID, "adjacency id >= nv");
       }
-      g->d_off = nullptr;
-      compact_graph(g, d_off_orig);
+    };
+    try {
+      g->device = device;
+      g->nv = nv;
+      g->ne = ne;
+      g->directed = directed;
+      load_side(offsets, adj, g->h_off, &d_off_orig, &g->d_adj);
+      if (directed) {
+        load_side(rev_offsets, rev_adj, g->h_roff, &d_roff_orig, &g->d_radj);
+        // the in-edge CSR must be the transpose: every vertex's in-degree (its
+        // occurrences in adj) equals its reverse row length, and vice versa
+        if (ne && (!degrees_match(g->d_adj, ne, g->h_roff, nv) || !degrees_match(g->d_radj, ne, g->h_off, nv)))
+          fail(IBFS_E_INVALID, "rev_offsets/rev_adj is not the transpose of offsets/adj");
+      }
+      unsigned long long *o = d_off_orig, *ro = d_roff_orig;
+      d_off_orig = d_roff_orig = nullptr;
+      compact_graph(g, o, ro);  // frees o and ro
       finish_graph(g);
     } catch (...) {
+      cudaFree(d_off_orig);
+      cudaFree(d_roff_orig);
       graph_release(g);
       throw;
     }
@@ -491,10 +584,11 @@ extern "C" int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const
     *out_graph = nullptr;
     if (nv == 0) fail(IBFS_E_INVALID, "nv must be >= 1");
     if (n_tuples > 0 && (!u || !v)) fail(IBFS_E_INVALID, "u/v is NULL");
-    if (directed) fail(IBFS_E_UNSUPPORTED, "directed graphs are not implemented in this build");
     if (n_tuples >= (1ull << 39)) fail(IBFS_E_INVALID, "too many tuples");
     DeviceScope ds(device);
-    const uint64_t ne = 2 * n_tuples;
+    // undirected: tuple (u, v) -> entries u->v and v->u; directed: u->v only, plus
+    // the in-edge rows v <- u for bottom-up
+    const uint64_t ne = directed ? n_tuples : 2 * n_tuples;
     ibfs_graph *g = new ibfs_graph();
     std::vector<void *> tmp;
     auto dalloc = [&](size_t bytes) {
@@ -503,52 +597,83 @@ extern "C" int ibfs_load_edges(int device, uint32_t nv, uint64_t n_tuples, const
       tmp.push_back(p);
       return p;
     };
+    auto dfree = [&](void *p) {
+      for (void *&q : tmp)
+        if (q == p) q = nullptr;
+      cudaFree(p);
+    };
+    int bits = 1;
+    while (bits < 32 && (1ull << bits) < nv) ++bits;
+    // rows of (key -> val) pairs: offsets = exclusive scan of the key histogram; a stable
+    // radix sort by key keeps tuple order within each row
+    auto build_rows = [&](const uint32_t *keys, const uint32_t *vals, uint64_t m, unsigned long long *off_out,
+                          uint32_t *adj_out) {
+      unsigned long long *deg = (unsigned long long *)dalloc(((size_t)nv + 1) * 8);
+      CK(cudaMemset(deg, 0, ((size_t)nv + 1) * 8));
+      if (m) {
+        count_ids_kernel<<<4096, 256>>>(keys, m, deg);
+        CK(cudaGetLastError());
+      }
+      size_t tb = 0;
+      CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, off_out, (int64_t)nv + 1));
+      void *t = dalloc(tb);
+      CK(cub::DeviceScan::ExclusiveSum(t, tb, deg, off_out, (int64_t)nv + 1));
+      if (m) {
+        uint32_t *keys_out = (uint32_t *)dalloc(m * 4);
+        size_t tb2 = 0;
+        CK(cub::DeviceRadixSort::SortPairs(nullptr, tb2, keys, keys_out, vals, adj_out, (int64_t)m, 0, bits));
+        void *t2 = dalloc(tb2);
+        CK(cub::DeviceRadixSort::SortPairs(t2, tb2, keys, keys_out, vals, adj_out, (int64_t)m, 0, bits));
+        CK(cudaDeviceSynchronize());
+        dfree(keys_out);
+        dfree(t2);
+      }
+      CK(cudaDeviceSynchronize());
+      dfree(deg);
+      dfree(t);
+    };
     try {
       g->device = device;
       g->nv = nv;
       g->ne = ne;
+      g->directed = directed != 0;
       uint32_t *d_u = (uint32_t *)dalloc(n_tuples * 4), *d_v = (uint32_t *)dalloc(n_tuples * 4);
       if (n_tuples) {
         CK(cudaMemcpy(d_u, u, n_tuples * 4, cudaMemcpyDefault));
         CK(cudaMemcpy(d_v, v, n_tuples * 4, cudaMemcpyDefault));
       }
-      uint32_t *keys_a = (uint32_t *)dalloc(ne * 4), *keys_b = (uint32_t *)dalloc(ne * 4);
-      uint32_t *vals_a = (uint32_t *)dalloc(ne * 4);
-      unsigned long long *deg = (unsigned long long *)dalloc(((size_t)nv + 1) * 8);
       uint32_t *bad = (uint32_t *)dalloc(4);
-      CK(cudaMemset(deg, 0, ((size_t)nv + 1) * 8));
       CK(cudaMemset(bad, 0, 4));
       if (n_tuples) {
-        explode_kernel<<<4096, 256>>>(d_u, d_v, n_tuples, keys_a, vals_a, deg, nv, bad);
+        check_ids_kernel<<<4096, 256>>>(d_u, d_v, n_tuples, nv, bad);
         CK(cudaGetLastError());
       }
       uint32_t hbad = 0;
       CK(cudaMemcpy(&hbad, bad, 4, cudaMemcpyDeviceToHost));
       if (hbad) fail(IBFS_E_INVALID, "tuple vertex id >= nv");
-      cudaFree(d_u);
-      cudaFree(d_v);
-      tmp[0] = tmp[1] = nullptr;
       unsigned long long *d_off_orig = (unsigned long long *)dalloc(((size_t)nv + 1) * sizeof(unsigned long long));
-      {  // offsets = exclusive scan of degrees (deg[nv] = 0 gives offsets[nv] = ne)
-        size_t tb = 0;
-        CK(cub::DeviceScan::ExclusiveSum(nullptr, tb, deg, d_off_orig, (int64_t)nv + 1));
-        void *t = dalloc(tb);
-        CK(cub::DeviceScan::ExclusiveSum(t, tb, deg, d_off_orig, (int64_t)nv + 1));
-      }
+      unsigned long long *d_roff_orig = nullptr;
       CK(cudaMalloc(&g->d_adj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
-      if (ne) {  // stable radix sort of (src, dst) by src keeps tuple order within rows
-        int bits = 1;
-        while (bits < 32 && (1ull << bits) < nv) ++bits;
-        size_t tb = 0;
-        CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, keys_a, keys_b, vals_a, g->d_adj, (int64_t)ne, 0, bits));
-        void *t = dalloc(tb);
-        CK(cub::DeviceRadixSort::SortPairs(t, tb, keys_a, keys_b, vals_a, g->d_adj, (int64_t)ne, 0, bits));
+      if (directed) {
+        d_roff_orig = (unsigned long long *)dalloc(((size_t)nv + 1) * sizeof(unsigned long long));
+        CK(cudaMalloc(&g->d_radj, std::max<uint64_t>(ne, 1) * sizeof(uint32_t)));
+        build_rows(d_u, d_v, n_tuples, d_off_orig, g->d_adj);   // out-edges u -> v
+        build_rows(d_v, d_u, n_tuples, d_roff_orig, g->d_radj); // in-edges v <- u
+      } else {
+        uint32_t *keys_a = (uint32_t *)dalloc(ne * 4), *vals_a = (uint32_t *)dalloc(ne * 4);
+        if (n_tuples) {
+          explode_kernel<<<4096, 256>>>(d_u, d_v, n_tuples, keys_a, vals_a);
+          CK(cudaGetLastError());
+        }
+        dfree(d_u);
+        dfree(d_v);
+        build_rows(keys_a, vals_a, ne, d_off_orig, g->d_adj);
       }
       CK(cudaDeviceSynchronize());
       for (void *&p : tmp)
-        if (p != d_off_orig) { cudaFree(p); p = nullptr; }
+        if (p && p != d_off_orig && p != d_roff_orig) { cudaFree(p); p = nullptr; }
       tmp.clear();
-      compact_graph(g, d_off_orig);  // frees d_off_orig
+      compact_graph(g, d_off_orig, d_roff_orig);  // frees both
       finish_graph(g);
     } catch (...) {
       for (void *p : tmp) cudaFree(p);
@@ -579,6 +704,12 @@ extern "C" int ibfs_graph_sort_rows(ibfs_graph *g, int order) {
     if (order != IBFS_ROWS_KEEP && order != IBFS_ROWS_HUB_FIRST) fail(IBFS_E_INVALID, "bad row order");
     if (order == IBFS_ROWS_KEEP || g->ne == 0) return;
     DeviceScope ds(g->device);
+    // the rows bottom-up scans: the in-edge rows of a directed graph, keyed
+    // by the in-degree of the parent (a vertex with many in-edges is reached early)
+    const std::vector<uint64_t> &h_off = g->directed ? g->h_roff : g->h_off;
+    const unsigned long long *d_off = g->directed ? g->d_roff : g->d_off;
+    uint32_t *d_adj = g->directed ? g->d_radj : g->d_adj;
+    const uint32_t *d_kdeg = g->directed ? g->d_rdeg : g->d_deg;
     // rows in batches of <= 2^30 entries (CUB segmented sort takes int sizes)
     const unsigned long long cap = 1ull << 30;
     unsigned long long maxb = 0;
@@ -586,10 +717,10 @@ extern "C" int ibfs_graph_sort_rows(ibfs_graph *g, int order) {
     uint32_t r0 = 0;
     while (r0 < g->nva) {
       uint32_t r1 = r0;
-      while (r1 < g->nva && g->h_off[r1 + 1] - g->h_off[r0] <= cap) ++r1;
+      while (r1 < g->nva && h_off[r1 + 1] - h_off[r0] <= cap) ++r1;
       if (r1 == r0) ++r1;  // a single row longer than cap (degree > 2^30): not expected
       batches.push_back({r0, r1});
-      maxb = std::max<unsigned long long>(maxb, g->h_off[r1] - g->h_off[r0]);
+      maxb = std::max<unsigned long long>(maxb, h_off[r1] - h_off[r0]);
       r0 = r1;
     }
     if (maxb > 0x7fffffffull) fail(IBFS_E_UNSUPPORTED, "row longer than 2^31 entries");
@@ -609,20 +740,20 @@ extern "C" int ibfs_graph_sort_rows(ibfs_graph *g, int order) {
       size_t tb_max = 0;
       for (auto &b : batches) {
         size_t tb = 0;
-        const int nitems = (int)(g->h_off[b.second] - g->h_off[b.first]);
+        const int nitems = (int)(h_off[b.second] - h_off[b.first]);
         const int nseg = (int)(b.second - b.first);
         CK(cub::DeviceSegmentedSort::StableSortPairs(nullptr, tb, kin, kout, vout, vout, nitems, nseg, rel, rel + 1));
         tb_max = std::max(tb_max, tb);
       }
       void *temp = dalloc(tb_max);
       for (auto &b : batches) {
-        const unsigned long long base = g->h_off[b.first];
-        const int nitems = (int)(g->h_off[b.second] - base);
+        const unsigned long long base = h_off[b.first];
+        const int nitems = (int)(h_off[b.second] - base);
         const int nseg = (int)(b.second - b.first);
         if (nitems == 0) continue;
-        uint32_t *vals = g->d_adj + base;
-        hubkey_kernel<<<4096, 256>>>(vals, g->d_deg, (unsigned long long)nitems, kin);
-        rel_offsets_kernel<<<(nseg + 256) / 256, 256>>>(g->d_off, b.first, (uint32_t)nseg, rel);
+        uint32_t *vals = d_adj + base;
+        hubkey_kernel<<<4096, 256>>>(vals, d_kdeg, (unsigned long long)nitems, kin);
+        rel_offsets_kernel<<<(nseg + 256) / 256, 256>>>(d_off, b.first, (uint32_t)nseg, rel);
         CK(cudaGetLastError());
         size_t tb = tb_max;
         CK(cub::DeviceSegmentedSort::StableSortPairs(temp, tb, kin, kout, vals, vout, nitems, nseg, rel, rel + 1));
@@ -876,7 +1007,8 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   T *ring = sc.get<T>((size_t)R * G * gstride);
   uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
-  uint32_t *chq = sc.get<uint32_t>((size_t)G * 2 * std::max<uint32_t>(g->n_chunks, 1));
+  const uint32_t chq_stride = std::max<uint32_t>(std::max(g->n_chunks, g->n_rchunks), 1);
+  uint32_t *chq = sc.get<uint32_t>((size_t)G * 2 * chq_stride);
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
   LevelStat *lstat = sc.get<LevelStat>((size_t)G * MAXL);
   uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
@@ -898,6 +1030,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.off = g->d_off;
   a.adj = g->d_adj;
   a.deg = g->d_deg;
+  a.directed = g->directed ? 1u : 0u;
+  a.roff = g->directed ? g->d_roff : g->d_off;
+  a.radj = g->directed ? g->d_radj : g->d_adj;
+  a.rdeg = g->directed ? g->d_rdeg : g->d_deg;
   a.tbase = g->d_tbase;
   a.nzbits = g->d_nzbits;
   a.nv = nv;
@@ -920,6 +1056,12 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.hub_vtx = g->d_hub_vtx;
   a.hub_chunk0 = g->d_hub_chunk0;
   a.n_hubs = g->n_hubs;
+  a.rchunks = g->directed ? g->d_rchunks : g->d_chunks;
+  a.n_rchunks = g->directed ? g->n_rchunks : g->n_chunks;
+  a.rhub_vtx = g->directed ? g->d_rhub_vtx : g->d_hub_vtx;
+  a.rhub_chunk0 = g->directed ? g->d_rhub_chunk0 : g->d_hub_chunk0;
+  a.n_rhubs = g->directed ? g->n_rhubs : g->n_hubs;
+  a.chq_stride = chq_stride;
   a.chq = chq;
   a.tdq = tdq;
   a.buq = buq;

@@ -102,9 +102,15 @@ struct Policy {
 
 template <typename T>
 struct BatchArgs {
-  const unsigned long long *off;  // compacted CSR (vertices of degree > 0 only)
-  const uint32_t *adj;
+  const unsigned long long *off;  // compacted CSR (vertices of degree > 0 only): out-edges
+  const uint32_t *adj;            // (top-down reads these rows)
   const uint32_t *deg;
+  // in-edge CSR for bottom-up ("directed graphs also store reverse edges"); for
+  // an undirected graph these alias off / adj / deg and the hub lists below
+  const unsigned long long *roff;
+  const uint32_t *radj;
+  const uint32_t *rdeg;
+  uint32_t directed;
   const uint32_t *tbase;   // [nv/128 + 1] non-isolated vertices before each 128-vertex tile
   const uint32_t *nzbits;  // [nv/32] bit v%32 of word v/32: vertex v has degree > 0
   uint32_t nv;     // vertices of the caller's graph (depth row length)
@@ -126,12 +132,18 @@ struct BatchArgs {
   const uint32_t *src;  // this batch's sources (caller ids), group-major, row g*W + j
   const uint32_t *csrc; // the same in compacted ids (NO_VERTEX if the source is isolated)
   int8_t *out;          // row g*W + j of this batch at out + (g*W + j) * nv
-  const HubChunk *chunks;
+  const HubChunk *chunks;       // out-edge rows of degree > HUB_T (top-down)
   uint32_t n_chunks;
   const uint32_t *hub_vtx;     // [n_hubs] compacted ids of the vertices of degree > HUB_T, ascending
   const uint32_t *hub_chunk0;  // [n_hubs + 1] first chunk of each hub (chunks are in hub order)
   uint32_t n_hubs;
-  uint32_t *chq;               // [gcap][2][n_chunks] hub-chunk queues (TD, BU)
+  const HubChunk *rchunks;     // the same for the in-edge rows (bottom-up)
+  uint32_t n_rchunks;
+  const uint32_t *rhub_vtx;
+  const uint32_t *rhub_chunk0;
+  uint32_t n_rhubs;
+  uint32_t chq_stride;         // max(n_chunks, n_rchunks)
+  uint32_t *chq;               // [gcap][2][chq_stride] hub-chunk queues (TD, BU)
   uint32_t *gbar;              // [2] grid barrier (count, generation)
   unsigned long long *tstamp;  // [MAXL][3] globaltimer: first CTA start, barrier, last CTA end
   uint32_t n_iso;       // vertices of degree 0 (nv - nva)
@@ -219,20 +231,23 @@ __device__ __forceinline__ void push_hub_chunks(const BatchArgs<T> &a, int g, ui
   uint32_t bal = __ballot_sync(FULL, pred);
   if (!bal) return;
   const int lane = threadIdx.x & 31;
-  uint32_t *q = a.chq + ((size_t)g * 2 + (cls - Q_TDC)) * a.n_chunks;
+  const bool bu = cls == Q_BUC;
+  uint32_t *q = a.chq + ((size_t)g * 2 + (cls - Q_TDC)) * a.chq_stride;
+  const uint32_t *hvtx = bu ? a.rhub_vtx : a.hub_vtx, *hc0 = bu ? a.rhub_chunk0 : a.hub_chunk0;
+  const uint32_t nh = bu ? a.n_rhubs : a.n_hubs;
   while (bal) {
     const int src = __ffs(bal) - 1;
     bal &= bal - 1;
     const uint32_t hv = __shfl_sync(FULL, v, src);
     uint32_t c0 = 0, c1 = 0, base = 0;
     if (lane == 0) {
-      uint32_t lo = 0, hi = a.n_hubs;  // hub index: binary search (hubs are few and sorted)
+      uint32_t lo = 0, hi = nh;  // hub index: binary search (hubs are few and sorted)
       while (hi - lo > 1) {
         const uint32_t mid = (lo + hi) >> 1;
-        if (__ldg(a.hub_vtx + mid) <= hv) lo = mid; else hi = mid;
+        if (__ldg(hvtx + mid) <= hv) lo = mid; else hi = mid;
       }
-      c0 = __ldg(a.hub_chunk0 + lo);
-      c1 = __ldg(a.hub_chunk0 + lo + 1);
+      c0 = __ldg(hc0 + lo);
+      c1 = __ldg(hc0 + lo + 1);
       base = atomicAdd(qlen + cls, c1 - c0);
     }
     c0 = __shfl_sync(FULL, c0, 0);
@@ -337,8 +352,8 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
       st(s1 + v, z);
     }
     if (first_dir) {
-      const uint32_t d = in ? __ldg(a.deg + v) : 0u;
-      const bool q = in && d <= (uint32_t)HUB_T;
+      const uint32_t d = in ? __ldg(a.rdeg + v) : 0u;  // bottom-up reads in-edge rows
+      const bool q = in && d > 0 && d <= (uint32_t)HUB_T;
       queue_push(a, g, qlen, Q_BUL, q && d <= (uint32_t)LIGHT_DEG, (uint32_t)v);
       queue_push(a, g, qlen, Q_BUH, q && d > (uint32_t)LIGHT_DEG, (uint32_t)v);
       push_hub_chunks(a, g, qlen, Q_BUC, in && d > (uint32_t)HUB_T, (uint32_t)v);
@@ -570,8 +585,8 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
     if (c_next < i1 && i < i1) {
       x_next = queue_at(a, q, cls, i);
       tx_next = wandn(active, ldg(vis + x_next));
-      dx_next = __ldg(a.deg + x_next);
-      ox_next = __ldg(a.off + x_next);
+      dx_next = __ldg(a.rdeg + x_next);
+      ox_next = __ldg(a.roff + x_next);
     } else {
       tx_next = wzero_value<T>();
       dx_next = 0;
@@ -615,7 +630,7 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
         has = true;
         proc++;
 #pragma unroll
-        for (int u = 0; u < 4; ++u) wn[u] = ((uint32_t)u < d) ? __ldg(a.adj + s0 + u) : 0xffffffffu;
+        for (int u = 0; u < 4; ++u) wn[u] = ((uint32_t)u < d) ? __ldg(a.radj + s0 + u) : 0xffffffffu;
       }
     }
     head += min((uint32_t)__popc(idle), avail);
@@ -634,7 +649,7 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       for (int u = 0; u < 4; ++u) x[u] = w[u] != 0xffffffffu ? ldg(vis + w[u]) : wzero_value<T>();
       k += 4;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) wn[u] = (k + u < d) ? __ldg(a.adj + s0 + k + u) : 0xffffffffu;
+      for (int u = 0; u < 4; ++u) wn[u] = (k + u < d) ? __ldg(a.radj + s0 + k + u) : 0xffffffffu;
 #pragma unroll
       for (int u = 0; u < 4; ++u)
         if (w[u] != 0xffffffffu) { acc = wor(acc, wand(x[u], tg)); insp++; }
@@ -711,7 +726,7 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
       for (int u = 0; u < U; ++u) {
         const unsigned long long e = e0 + u * BLOCK + tid;
         if (e < c.e1) {
-          const uint32_t w = __ldg(a.adj + e);
+          const uint32_t w = __ldg(a.radj + e);
           x = wor(x, wand(ldg(vis + w), tg));
           insp++;
         }
@@ -791,7 +806,8 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     const T all = wnot(wzero_value<T>());
     const bool filt = ldcg(&c->td_filter) != 0;
     if (ph == 0) {
-      const HubChunk hc = a.chunks[a.chq[((size_t)g * 2 + d) * a.n_chunks + k]];
+      const uint32_t ci = a.chq[((size_t)g * 2 + d) * a.chq_stride + k];
+      const HubChunk hc = d ? a.rchunks[ci] : a.chunks[ci];
       if (d == 0) hub_td<T>(a, sm, g, hc, level, filt, bu_level ? td_bits : all);
       else hub_bu<T>(a, sm, s_red, g, hc, level, ldcg_w(&c->active), td_bits);
       continue;
@@ -886,17 +902,18 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
   uint32_t *qlen = c->qlen[lc & 1];
   const size_t nv = a.nva;
   T n[CVT], vv[CVT];
-  uint32_t dg[CVT];
+  uint32_t dg[CVT], rdg[CVT];  // out-degree (top-down rows), in-degree (bottom-up rows)
 #pragma unroll
   for (int k = 0; k < CVT; ++k) {
     const size_t v = base + (size_t)k * BLOCK + tid;
     n[k] = wzero_value<T>();
     vv[k] = wzero_value<T>();
-    dg[k] = 0;
+    dg[k] = rdg[k] = 0;
     if (v < nv) {
       n[k] = ld(N + v);
       vv[k] = ld(vis + v);
       dg[k] = __ldg(a.deg + v);
+      rdg[k] = a.directed ? __ldg(a.rdeg + v) : dg[k];
     }
   }
   uint32_t bal[CVT][4];
@@ -915,23 +932,27 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
     if (nz) st(vis + v, wor(vv[k], n[k]));
     const T tp = in ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
     const bool un = !wzero(tp);
-    const uint32_t d = dg[k];
+    const uint32_t d = dg[k], rd = rdg[k];
     if (nz) {
       nf++;
       mf += d;
       newp += wpopc(n[k]);
       nacc = wor(nacc, n[k]);
     }
+    // top-down classes by out-degree, bottom-up classes by in-degree (a vertex without
+    // in-edges can never be found bottom-up and is not queued)
     const bool qd = d > 0 && d <= (uint32_t)HUB_T;
     const bool light = d <= (uint32_t)LIGHT_DEG;
+    const bool rqd = rd > 0 && rd <= (uint32_t)HUB_T;
+    const bool rlight = rd <= (uint32_t)LIGHT_DEG;
     bal[k][Q_TDL] = __ballot_sync(FULL, nz && qd && light);
     bal[k][Q_TDH] = __ballot_sync(FULL, nz && qd && !light);
-    bal[k][Q_BUL] = __ballot_sync(FULL, un && qd && light);
-    bal[k][Q_BUH] = __ballot_sync(FULL, un && qd && !light);
+    bal[k][Q_BUL] = __ballot_sync(FULL, un && rqd && rlight);
+    bal[k][Q_BUH] = __ballot_sync(FULL, un && rqd && !rlight);
     // hubs: their chunks, never the vertex queues (rare: one vote in the common case)
-    if (__any_sync(FULL, in && d > (uint32_t)HUB_T)) {
+    if (__any_sync(FULL, in && (d > (uint32_t)HUB_T || rd > (uint32_t)HUB_T))) {
       push_hub_chunks(a, g, qlen, Q_TDC, in && nz && d > (uint32_t)HUB_T, (uint32_t)v);
-      push_hub_chunks(a, g, qlen, Q_BUC, in && un && d > (uint32_t)HUB_T, (uint32_t)v);
+      push_hub_chunks(a, g, qlen, Q_BUC, in && un && rd > (uint32_t)HUB_T, (uint32_t)v);
     }
 #pragma unroll
     for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);

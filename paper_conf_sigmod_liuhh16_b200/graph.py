@@ -123,17 +123,24 @@ class Graph:
         return self
 
     @classmethod
-    def from_csr(cls, offsets, adj, device: int = 0) -> "Graph":
+    def from_csr(cls, offsets, adj, device: int = 0, rev_offsets=None, rev_adj=None) -> "Graph":
+        """ibfs_load_csr.  Directed graphs also pass the in-edge CSR (rev_offsets, rev_adj)."""
         lib = _lib.load()
         if isinstance(offsets, np.ndarray):
             offsets = np.ascontiguousarray(offsets, dtype=np.uint64)
             adj = np.ascontiguousarray(adj, dtype=np.uint32)
+        if isinstance(rev_offsets, np.ndarray):
+            rev_offsets = np.ascontiguousarray(rev_offsets, dtype=np.uint64)
+            rev_adj = np.ascontiguousarray(rev_adj, dtype=np.uint32)
         po, ko = _ptr(offsets)
         pa, ka = _ptr(adj)
+        pro, kro = _ptr(rev_offsets)
+        pra, kra = _ptr(rev_adj)
         nv = _len(offsets) - 1
         ne = _len(adj)
         h = C.c_void_p()
-        check(lib.ibfs_load_csr(int(device), nv, ne, po, pa if ne else None, None, None, C.byref(h)))
+        check(lib.ibfs_load_csr(int(device), nv, ne, po, pa if ne else None, pro,
+                                pra if (ne and pro) else None, C.byref(h)))
         return cls(h, device)
 
     @classmethod

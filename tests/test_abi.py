@@ -83,10 +83,11 @@ def test_validation_before_device_work(lib):
     adj = np.array([1, 0], dtype=np.uint32)
     assert lib.ibfs_load_csr(0, 2, 2, off.ctypes.data, adj.ctypes.data, None, None, None) == _lib.IBFS_E_INVALID
     assert lib.ibfs_load_csr(0, 0, 0, off.ctypes.data, None, None, None, C.byref(h)) == _lib.IBFS_E_INVALID
-    assert lib.ibfs_load_csr(0, 2, 2, off.ctypes.data, adj.ctypes.data, off.ctypes.data, adj.ctypes.data,
-                             C.byref(h)) == _lib.IBFS_E_UNSUPPORTED
+    # directed: the in-edge CSR comes as a pair
+    assert lib.ibfs_load_csr(0, 2, 2, off.ctypes.data, adj.ctypes.data, off.ctypes.data, None,
+                             C.byref(h)) == _lib.IBFS_E_INVALID
     assert lib.ibfs_load_edges(0, 2, 1, None, None, 0, C.byref(h)) == _lib.IBFS_E_INVALID
-    assert lib.ibfs_load_edges(0, 2, 1, adj.ctypes.data, adj.ctypes.data, 1, C.byref(h)) == _lib.IBFS_E_UNSUPPORTED
+    assert lib.ibfs_load_edges(0, 2, 1, None, None, 1, C.byref(h)) == _lib.IBFS_E_INVALID
     src = np.zeros(4, dtype=np.uint32)
     assert lib.ibfs_run(None, src.ctypes.data, 4, 64, None) == _lib.IBFS_E_INVALID
     assert lib.ibfs_run_ex(None, src.ctypes.data, 4, 64, None, None, None) == _lib.IBFS_E_INVALID

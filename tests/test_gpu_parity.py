@@ -237,7 +237,7 @@ def test_full_size_sampled_rows(name, rows):
 # ----------------------------------------------------------------------- planner
 @pytest.mark.parametrize("W", [32, 64, 128])
 def test_planner_matches_oracle_planner(W):
-    for cfg in (ibfs_gen.CONFIGS["c1"], ibfs_gen.CONFIGS["c2"]):
+    for cfg in (ibfs_gen.CONFIGS["c1"], ibfs_gen.CONFIGS["c2"], ibfs_gen.CONFIGS["d2"]):
         el = cfg.edges()
         src = cfg.sources(el)
         g = P.Graph.from_edgelist(el)
@@ -381,3 +381,86 @@ def test_khop_invalid():
     g = P.Graph.from_edgelist(ibfs_gen.from_pairs(4, [(0, 1)]))
     with pytest.raises(ValueError):
         g.run(np.array([0], dtype=np.uint32), 32, max_depth=0)
+
+
+# ------------------------------------------------------------ directed graphs (NEXT #1)
+# "for directed graphs, we also store the reverse edges" -- top-down expands the
+# out-edge rows, bottom-up reads a vertex's parents from the in-edge rows.  The oracle
+# runs its textbook BFS over out-edges (oracle.c, pinned by directed Floyd-Warshall).
+def _transpose_csr(nv, off, adj):
+    src = np.repeat(np.arange(nv, dtype=np.uint32), np.diff(off).astype(np.int64))
+    order = np.argsort(adj, kind="stable")
+    roff = np.zeros(nv + 1, dtype=np.uint64)
+    np.cumsum(np.bincount(adj, minlength=nv), out=roff[1:])
+    return roff, src[order]
+
+
+def test_directed_random_tiny_forced_schedules():
+    rng = np.random.default_rng(4242)
+    for trial in range(120):
+        nv = int(rng.integers(1, 60))
+        m = int(rng.integers(0, 4 * nv + 1))
+        pairs = [(int(rng.integers(nv)), int(rng.integers(nv))) for _ in range(m)]
+        if m:
+            pairs += [pairs[0], (pairs[-1][0], pairs[-1][0])]
+        el = ibfs_gen.from_pairs(nv, pairs if pairs else np.zeros((0, 2)), directed=True)
+        n = int(rng.integers(1, 3 * 64))
+        src = rng.integers(0, nv, size=n).astype(np.uint32)
+        W = int(rng.choice([32, 64, 128]))
+        kind = SCHEDULES[trial % len(SCHEDULES)]
+        split = ["auto", "off", "force"][trial % 3]
+        g = P.Graph.from_edgelist(el, hub_first=bool(trial % 2))
+        d, st = gpu_depths(g, src, W, split=split, split_mod=int(rng.integers(1, 6)), want_digest=True,
+                           **run_kwargs(kind, rng))
+        ref = oracle.bfs(el, src)
+        np.testing.assert_array_equal(d, ref.depths, err_msg=f"trial {trial} W={W} {kind} split={split}")
+        np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+        np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+
+
+@pytest.mark.parametrize("W", [32, 64, 128])
+@pytest.mark.parametrize("kind", ["auto", "td", "bu2"])
+def test_directed_config_full(W, kind):
+    cfg = ibfs_gen.CONFIGS["d2"]
+    el = cfg.edges()
+    assert el.directed
+    src = cfg.sources(el)
+    g = P.Graph.from_edgelist(el)
+    s = src[g.plan(src, W)]
+    d, st = gpu_depths(g, s, W, want_digest=True, **run_kwargs(kind))
+    key = ("d2", s.tobytes())
+    if key not in _C2:
+        _C2[key] = oracle.bfs(el, s)
+    ref = _C2[key]
+    np.testing.assert_array_equal(d, ref.depths)
+    np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+    np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+    # a directed graph is not symmetric: some pair must differ from the undirected BFS
+    und = _oracle_c2(ibfs_gen.CONFIGS["c2"].edges(), s) if W == 128 and kind == "auto" else None
+    if und is not None:
+        assert not np.array_equal(und.depths, d)
+
+
+def test_directed_from_csr_matches_from_edges_and_khop():
+    cfg = ibfs_gen.CONFIGS["d2"]
+    el = cfg.edges()
+    og = oracle.OracleGraph.from_edges(el)
+    off, adj = og.adjacency()
+    roff, radj = _transpose_csr(el.nv, off, adj)
+    g = P.Graph.from_csr(off, adj, rev_offsets=roff, rev_adj=radj)
+    src = cfg.sources(el)[:128]
+    d, st = gpu_depths(g, src, 128, want_digest=True)
+    ref = og.bfs(src)
+    np.testing.assert_array_equal(d, ref.depths)
+    np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+    d3, _ = gpu_depths(g, src, 128, max_depth=3)
+    np.testing.assert_array_equal(d3, og.bfs(src, max_depth=3).depths)
+    # the out-edge rows come back unchanged
+    eo, ea = g.export_csr()
+    np.testing.assert_array_equal(eo, off)
+    np.testing.assert_array_equal(ea, adj)
+    # a reverse CSR that is not the transpose is rejected
+    bad_off = roff.copy()
+    bad_off[1:-1] = np.minimum(bad_off[1:-1] + 1, bad_off[-1])
+    with pytest.raises(Exception):
+        P.Graph.from_csr(off, adj, rev_offsets=bad_off, rev_adj=radj)

@@ -34,3 +34,16 @@ def build(force: bool = False, verbose: bool = False) -> str:
             cmd.insert(1, "-Xptxas=-v")
         subprocess.check_call(cmd, cwd=CSRC)
     return SO
+
+
+def build_variant(name: str, defines: dict) -> str:
+    """A/B build (tuning experiments): build/libibfs_<name>.so with -D overrides of the
+    compile-time knobs (IBFS_EXPAND_MINB, IBFS_BU_U); select it with IBFS_LIB=<path>."""
+    out_dir = os.path.join(os.path.dirname(HERE), "build")
+    os.makedirs(out_dir, exist_ok=True)
+    out = os.path.join(out_dir, f"libibfs_{name}.so")
+    nvcc = os.environ.get("NVCC", "nvcc")
+    cmd = [nvcc, *NVCC_FLAGS, *[f"-D{k}={v}" for k, v in defines.items()], "-o", out] + \
+        [os.path.join(CSRC, f) for f in SOURCES]
+    subprocess.check_call(cmd, cwd=CSRC)
+    return out

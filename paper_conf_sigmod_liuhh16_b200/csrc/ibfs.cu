@@ -1007,6 +1007,8 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   T *ring = sc.get<T>((size_t)R * G * gstride);
   uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
+  const uint32_t nchunk32 = (nva + 31) / 32;
+  uint8_t *dirty = sc.get<uint8_t>((size_t)G * std::max<uint32_t>(nchunk32, 1));
   const uint32_t chq_stride = std::max<uint32_t>(std::max(g->n_chunks, g->n_rchunks), 1);
   uint32_t *chq = sc.get<uint32_t>((size_t)G * 2 * chq_stride);
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
@@ -1065,6 +1067,8 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.chq = chq;
   a.tdq = tdq;
   a.buq = buq;
+  a.dirty = dirty;
+  a.nchunk32 = nchunk32;
   a.n_iso = nv - nva;
   a.pol.mode = o.direction;
   a.pol.bu_from = o.bu_from;

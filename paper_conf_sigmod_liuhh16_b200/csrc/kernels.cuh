@@ -50,6 +50,10 @@ constexpr unsigned FULL = 0xffffffffu;
 #ifndef IBFS_EXPAND_MINB
 #define IBFS_EXPAND_MINB 3  // min resident expand CTAs per SM (register cap)
 #endif
+#ifndef IBFS_BU_U
+#define IBFS_BU_U 4  // neighbours a bottom-up thread inspects per step (loads in flight)
+#endif
+constexpr int BU_U = IBFS_BU_U;
 
 // queue classes
 constexpr int Q_TDL = 0, Q_TDH = 1, Q_BUL = 2, Q_BUH = 3;
@@ -83,6 +87,10 @@ struct GroupCtrl {
   // per-instance direction split of a bottom-up level (include/ibfs.h IBFS_SPLIT_*):
   // td_bits = the active instances expanded top-down in the next level when dir == BU
   T td_bits;
+  // sparse commit after a small top-down level: 32-vertex chunks of S_l written by the
+  // level's top-down part (approximate count, [parity of the level])
+  uint32_t ndirty[2];
+  uint32_t sparse;  // the last commit was sparse (no bottom-up queue: the next level is TD)
   float bitw[WordBits<T>::value];  // sampled degree sum of the new frontier per instance (commit)
   float cumw[WordBits<T>::value];  // running sum of bitw over the levels so far (visited edges)
 };
@@ -121,6 +129,8 @@ struct BatchArgs {
   int R;         // ring slots
   int gcap;      // groups allocated per slot
   uint32_t *tdq, *buq;  // [gcap][nva] queues
+  uint8_t *dirty;       // [gcap][nchunk32] 32-vertex chunk of S_l written by a top-down RED.OR
+  uint32_t nchunk32;    // ceil(nva / 32)
   GroupCtrl<T> *ctrl;
   LevelStat *lstat;     // [G][MAXL]
   uint32_t *work_ctr;   // [MAXL]
@@ -179,6 +189,17 @@ __device__ __forceinline__ uint32_t *queue_of(const BatchArgs<T> &a, int g, int 
 template <typename T>
 __device__ __forceinline__ uint32_t queue_at(const BatchArgs<T> &a, const uint32_t *q, int cls, uint32_t i) {
   return (cls & 1) ? q[a.nva - 1 - i] : q[i];
+}
+
+// Top-down write to vertex w of group g: mark its 32-vertex chunk for the sparse commit
+// (plain byte stores; the count of newly marked chunks is approximate under races).
+template <typename T>
+__device__ __forceinline__ void mark_dirty(const BatchArgs<T> &a, int g, uint32_t w, uint32_t &ndirty) {
+  uint8_t *f = a.dirty + (size_t)g * a.nchunk32 + (w >> 5);
+  if (!*(volatile uint8_t *)f) {
+    *f = 1;
+    ndirty++;
+  }
 }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -305,6 +326,8 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     c.arrive = 0;
     c.last_level = done ? 0xffffffffu : 0u;  // done at init: no snapshot was ever written
     c.td_bits = wzero_value<T>();
+    c.ndirty[0] = c.ndirty[1] = 0;
+    c.sparse = 0;
     for (int j = 0; j < W; ++j) c.bitw[j] = c.cumw[j] = 0.f;
     a.ctrl[g] = c;
     if (rows > 0) {
@@ -350,6 +373,7 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
       st(vis + v, z);
       st(s0 + v, z);
       st(s1 + v, z);
+      if ((v & 31) == 0) a.dirty[(size_t)g * a.nchunk32 + (v >> 5)] = 0;
     }
     if (first_dir) {
       const uint32_t d = in ? __ldg(a.rdeg + v) : 0u;  // bottom-up reads in-edge rows
@@ -481,6 +505,12 @@ __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq
   }
 }
 
+template <typename T>
+__device__ __forceinline__ void flush_dirty(const BatchArgs<T> &a, int g, int level, uint32_t ndirty) {
+  ndirty = __reduce_add_sync(FULL, ndirty);
+  if ((threadIdx.x & 31) == 0 && ndirty) atomicAdd(&a.ctrl[g].ndirty[level & 1], ndirty);
+}
+
 // Top-down item: entries [i0, i1) of a TD queue class.  The frontier words and rows of
 // the entries are staged in shared memory, then an edge-balanced sweep (load-balanced
 // search on the degree prefix) ORs each frontier word into its unvisited neighbours
@@ -496,7 +526,7 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
   const T *vis = a.visited + (size_t)g * a.gstride;
   const uint32_t *q = queue_of(a, g, cls);
   const uint32_t qn = i1 - i0;
-  uint32_t insp = 0, writes = 0;
+  uint32_t insp = 0, writes = 0, ndirty = 0;
   for (uint32_t i = tid; i < qn; i += BLOCK) {
     const uint32_t v = queue_at(a, q, cls, i0 + i);
     const T f = wand(ldg(F + v), fmask);
@@ -526,11 +556,12 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       if (w[u] != 0xffffffffu) {
         insp++;
         const T b = filt ? wandn(fw[u], ldg(vis + w[u])) : fw[u];
-        if (!wzero(b)) { red_or(N + w[u], b); writes++; }
+        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u], ndirty); }
       }
     }
   }
   flush_counts(sm, g, 0u, 0u, tid == 0 ? qn : 0u, insp, writes);
+  flush_dirty(a, g, level, ndirty);
 }
 
 // Bottom-up item: entries [i0, i1) of a BU queue class.
@@ -573,7 +604,7 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
   uint32_t v = 0, d = 0, k = 0;
   unsigned long long s0 = 0;
   T tg = wzero_value<T>(), acc = wzero_value<T>();
-  uint32_t wn[4];  // adjacency entries of the lane's next step (prefetched)
+  uint32_t wn[BU_U];  // adjacency entries of the lane's next step (prefetched)
   // refill pipeline: the loads for the next 32 queue entries are issued one round early
   uint32_t c_next = 0, x_next = 0, dx_next = 0;
   T tx_next = wzero_value<T>();
@@ -630,7 +661,7 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
         has = true;
         proc++;
 #pragma unroll
-        for (int u = 0; u < 4; ++u) wn[u] = ((uint32_t)u < d) ? __ldg(a.radj + s0 + u) : 0xffffffffu;
+        for (int u = 0; u < BU_U; ++u) wn[u] = ((uint32_t)u < d) ? __ldg(a.radj + s0 + u) : 0xffffffffu;
       }
     }
     head += min((uint32_t)__popc(idle), avail);
@@ -641,17 +672,17 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       continue;
     }
     if (has) {
-      uint32_t w[4];
+      uint32_t w[BU_U];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) w[u] = wn[u];
-      T x[4];
+      for (int u = 0; u < BU_U; ++u) w[u] = wn[u];
+      T x[BU_U];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) x[u] = w[u] != 0xffffffffu ? ldg(vis + w[u]) : wzero_value<T>();
-      k += 4;
+      for (int u = 0; u < BU_U; ++u) x[u] = w[u] != 0xffffffffu ? ldg(vis + w[u]) : wzero_value<T>();
+      k += BU_U;
 #pragma unroll
-      for (int u = 0; u < 4; ++u) wn[u] = (k + u < d) ? __ldg(a.radj + s0 + k + u) : 0xffffffffu;
+      for (int u = 0; u < BU_U; ++u) wn[u] = (k + u < d) ? __ldg(a.radj + s0 + k + u) : 0xffffffffu;
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+      for (int u = 0; u < BU_U; ++u)
         if (w[u] != 0xffffffffu) { acc = wor(acc, wand(x[u], tg)); insp++; }
       if (weq(acc, tg) || k >= d) {
         if (!wzero(acc)) {
@@ -675,7 +706,7 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
   const T *vis = a.visited + (size_t)g * a.gstride;
   const T f = wand(ldg(F + c.v), fmask);
   if (wzero(f)) return;
-  uint32_t insp = 0, writes = 0;
+  uint32_t insp = 0, writes = 0, ndirty = 0;
   constexpr int U = 8;
   for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
     uint32_t w[U];
@@ -689,12 +720,13 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
       if (w[u] != 0xffffffffu) {
         insp++;
         const T b = filt ? wandn(f, ldg(vis + w[u])) : f;
-        if (!wzero(b)) { red_or(N + w[u], b); writes++; }
+        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u], ndirty); }
       }
     }
   }
   const bool first = c.first && tid == 0;
   flush_counts(sm, g, 0u, 0u, first ? 1u : 0u, insp, writes);
+  flush_dirty(a, g, level, ndirty);
 }
 
 // Hub chunk, bottom-up: the CTA ORs a chunk of the hub's neighbours in waves, with a
@@ -888,11 +920,30 @@ constexpr int CVT = 4;
 constexpr int CTILE = CVT * BLOCK;  // vertices per commit tile
 constexpr int SAMPLE = SAMPLE_TILES * CVT;
 
+// Sparse commit of level lc: after a pure top-down level whose writes
+// touched at most a quarter of the 32-vertex chunks, the commit reads S_l / visited /
+// degrees only in the chunks marked dirty (every other chunk of S_l is zero: nothing new
+// there) and builds no bottom-up queue, so the next level must run top-down -- allowed
+// in auto mode (the override is a performance choice, never a result change) and in a
+// forced schedule only where that schedule says top-down.  Evaluated identically by
+// every CTA from state fixed before this launch.
+template <typename T>
+__device__ __forceinline__ bool commit_sparse(const BatchArgs<T> &a, const GroupCtrl<T> *c, int lc) {
+  if (c->dir != 0) return false;
+  if ((unsigned long long)c->ndirty[lc & 1] * 4ull > (unsigned long long)a.nchunk32) return false;
+  const uint32_t next = (uint32_t)lc + 1;
+  switch (a.pol.mode) {
+    case 0: case 1: return true;
+    case 2: return next < a.pol.bu_from;
+    default: return next - 1 < a.pol.sched_len ? a.pol.sched[next - 1] == 0 : true;
+  }
+}
+
 template <typename T>
 __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, size_t base,
                                             unsigned long long &nf, unsigned long long &mf,
                                             unsigned long long &newp, T &nacc, bool sample,
-                                            float (&bc)[WordBits<T>::value / 32]) {
+                                            float (&bc)[WordBits<T>::value / 32], bool sparse) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   GroupCtrl<T> *c = a.ctrl + g;
   const T active = c->active;
@@ -903,13 +954,19 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
   const size_t nv = a.nva;
   T n[CVT], vv[CVT];
   uint32_t dg[CVT], rdg[CVT];  // out-degree (top-down rows), in-degree (bottom-up rows)
+  bool live[CVT];              // chunk to read (dense commit, or marked dirty)
+  uint8_t *dfl = a.dirty + (size_t)g * a.nchunk32;
 #pragma unroll
   for (int k = 0; k < CVT; ++k) {
     const size_t v = base + (size_t)k * BLOCK + tid;
     n[k] = wzero_value<T>();
     vv[k] = wzero_value<T>();
     dg[k] = rdg[k] = 0;
-    if (v < nv) {
+    const size_t ch = (base + (size_t)k * BLOCK + (size_t)(warp * 32)) >> 5;  // warp-uniform chunk
+    const uint8_t fl = ch < a.nchunk32 ? dfl[ch] : (uint8_t)0;
+    if (fl && lane == 0) dfl[ch] = 0;  // consumed by this commit
+    live[k] = !sparse || fl;
+    if (v < nv && live[k]) {
       n[k] = ld(N + v);
       vv[k] = ld(vis + v);
       dg[k] = __ldg(a.deg + v);
@@ -930,7 +987,7 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
     }
     const bool nz = !wzero(n[k]);
     if (nz) st(vis + v, wor(vv[k], n[k]));
-    const T tp = in ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
+    const T tp = (in && !sparse) ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
     const bool un = !wzero(tp);
     const uint32_t d = dg[k], rd = rdg[k];
     if (nz) {
@@ -957,7 +1014,7 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
 #pragma unroll
     for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
   }
-  if (sample) {  // block-uniform
+  if (sample && !sparse) {  // block-uniform
     const uint32_t d0 = wzero(n[0]) ? 0u : dg[0];
     const uint32_t dmax = __reduce_or_sync(FULL, d0);
     if (dmax) {
@@ -1008,7 +1065,8 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
 template <typename T>
 __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, uint32_t ntiles,
                              uint32_t tiles_per_group, unsigned long long nf, unsigned long long mf,
-                             unsigned long long newp, T nacc, float (&bc)[WordBits<T>::value / 32]) {
+                             unsigned long long newp, T nacc, float (&bc)[WordBits<T>::value / 32],
+                             bool sparse) {
   constexpr int W = WordBits<T>::value;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   GroupCtrl<T> *c = a.ctrl + g;
@@ -1082,7 +1140,7 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     ls->nf = n_f;
     bool bu;
     T tdb = wzero_value<T>();
-    bu = decide_bu(a.pol, (uint32_t)lc + 1, cur, n_f, m_f);
+    bu = !sparse && decide_bu(a.pol, (uint32_t)lc + 1, cur, n_f, m_f);
     if (bu) {
       tdb = wfrom_pieces<T>(cm.tdb);
       // auto: if every active instance is small the level is plain top-down
@@ -1099,6 +1157,8 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->vpairs += np;
     c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
+    c->ndirty[lc & 1] = 0;
+    c->sparse = sparse ? 1u : 0u;
     c->last_level = (uint32_t)lc;
     for (int k = 0; k < NQ; ++k) c->qlen[(lc + 1) & 1][k] = 0;  // target of commit lc+1
     if (wzero(act) || (a.pol.max_depth != 0 && (uint32_t)lc >= a.pol.max_depth)) {
@@ -1176,6 +1236,7 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
     const uint32_t tpg = (uint32_t)((a.nva + CTILE - 1) / CTILE);
     const size_t total = (size_t)a.G * tpg;
     int cur_g = -1;
+    bool sparse = false;
     uint32_t ntiles = 0;
     unsigned long long nf = 0, mf = 0, newp = 0;
     T nacc = wzero_value<T>();
@@ -1188,18 +1249,19 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
     for (size_t w = blockIdx.x; w < total; w += gridDim.x) {
       const int g = (int)(w / tpg);
       if (g != cur_g) {
-        if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc);
+        if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc, sparse);
         cur_g = g;
+        sparse = !a.ctrl[g].done && commit_sparse(a, a.ctrl + g, lc);
         ntiles = 0;
         nf = mf = newp = 0;
         nacc = wzero_value<T>();
       }
       if (a.ctrl[g].done) continue;  // finished before this launch (stable)
       const uint32_t tix = (uint32_t)(w % tpg);
-      commit_tile(a, cm, g, lc, (size_t)tix * CTILE, nf, mf, newp, nacc, tix % SAMPLE_TILES == 0, bc);
+      commit_tile(a, cm, g, lc, (size_t)tix * CTILE, nf, mf, newp, nacc, tix % SAMPLE_TILES == 0, bc, sparse);
       ++ntiles;
     }
-    if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc);
+    if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc, sparse);
     grid_barrier(a.gbar);
   }
   if (tid == 0 && blockIdx.x == 0) {
@@ -1587,12 +1649,23 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
     uint32_t m[NP];
 #pragma unroll
     for (int p = 0; p < NP; ++p) m[p] = warp_transpose32(wpiece(x, p));
-    const uint32_t dmax = __reduce_or_sync(FULL, d);
-    const int nb = 32 - __clz(dmax);
+    // degrees < 256 through their 8 bit planes; the few larger ones (hubs) one by one
+    const bool heavy = d >= 256u;
+    const uint32_t dl = heavy ? 0u : d;
+    const int nb = 32 - __clz(__reduce_or_sync(FULL, dl));
     for (int b = 0; b < nb; ++b) {
-      const uint32_t db = __ballot_sync(FULL, (d >> b) & 1u);
+      const uint32_t db = __ballot_sync(FULL, (dl >> b) & 1u);
 #pragma unroll
       for (int p = 0; p < NP; ++p) acc[p] += (unsigned long long)__popc(m[p] & db) << b;
+    }
+    uint32_t hv = __ballot_sync(FULL, heavy && !wzero(x));
+    while (hv) {
+      const int src = __ffs(hv) - 1;
+      hv &= hv - 1;
+      const unsigned long long dd = __shfl_sync(FULL, d, src);
+#pragma unroll
+      for (int p = 0; p < NP; ++p)
+        if ((__shfl_sync(FULL, wpiece(x, p), src) >> lane) & 1u) acc[p] += dd;
     }
   }
 #pragma unroll

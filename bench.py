@@ -44,10 +44,12 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c5", choices=sorted(ibfs_gen.CONFIGS))
     ap.add_argument("--groups-per-rank", type=int, default=0)
+    ap.add_argument("--groups-in-flight", type=int, default=0, help="groups per launch batch (0 = library auto)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--direction", default="auto")
     ap.add_argument("--alpha", type=float, default=4.0)
     ap.add_argument("--beta", type=float, default=24.0)
+    ap.add_argument("--split-div", type=float, default=64.0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sources (0 = host cores)")
@@ -189,7 +191,8 @@ def main():
 
     out_dev = torch.empty((G * W, g.nv), dtype=torch.int8, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if args.config in ("c1", "c2", "c4") else None
-    run_kw = dict(direction=args.direction, alpha=args.alpha, beta=args.beta)
+    run_kw = dict(direction=args.direction, alpha=args.alpha, beta=args.beta, groups_in_flight=args.groups_in_flight,
+                  split_div=args.split_div)
     stream = torch.cuda.current_stream(dev)
 
     def do_step(k, timing):
@@ -300,6 +303,7 @@ def main():
                        "scale": cfg.scale, "edgefactor": cfg.ef, "group_bits": W,
                        "sources_per_rank_per_step": G * W, "groups_per_rank_per_step": G,
                        "planner": "GroupBy", "direction": args.direction,
+                       "groups_in_flight": args.groups_in_flight or "auto",
                        "l2": ("flush 256 MiB between steps" if flush is not None
                               else "inputs > L2 (adjacency + per-group state), no flush"),
                        "parallelism": f"groups sharded over {world} rank(s), graph replicated"},

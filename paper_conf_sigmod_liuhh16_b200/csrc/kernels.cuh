@@ -87,10 +87,7 @@ struct GroupCtrl {
   // per-instance direction split of a bottom-up level (include/ibfs.h IBFS_SPLIT_*):
   // td_bits = the active instances expanded top-down in the next level when dir == BU
   T td_bits;
-  // sparse commit after a small top-down level: 32-vertex chunks of S_l written by the
-  // level's top-down part (approximate count, [parity of the level])
-  uint32_t ndirty[2];
-  uint32_t sparse;  // the last commit was sparse (no bottom-up queue: the next level is TD)
+  uint32_t sparse;  // the last commit was sparse (no bottom-up queue: the next level is TD)  // the last commit was sparse (no bottom-up queue: the next level is TD)
   float bitw[WordBits<T>::value];  // sampled degree sum of the new frontier per instance (commit)
   float cumw[WordBits<T>::value];  // running sum of bitw over the levels so far (visited edges)
 };
@@ -192,14 +189,10 @@ __device__ __forceinline__ uint32_t queue_at(const BatchArgs<T> &a, const uint32
 }
 
 // Top-down write to vertex w of group g: mark its 32-vertex chunk for the sparse commit
-// (plain byte stores; the count of newly marked chunks is approximate under races).
+// (a fire-and-forget byte store; the level's write count bounds the marked chunks).
 template <typename T>
-__device__ __forceinline__ void mark_dirty(const BatchArgs<T> &a, int g, uint32_t w, uint32_t &ndirty) {
-  uint8_t *f = a.dirty + (size_t)g * a.nchunk32 + (w >> 5);
-  if (!*(volatile uint8_t *)f) {
-    *f = 1;
-    ndirty++;
-  }
+__device__ __forceinline__ void mark_dirty(const BatchArgs<T> &a, int g, uint32_t w) {
+  a.dirty[(size_t)g * a.nchunk32 + (w >> 5)] = 1;
 }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -326,7 +319,6 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     c.arrive = 0;
     c.last_level = done ? 0xffffffffu : 0u;  // done at init: no snapshot was ever written
     c.td_bits = wzero_value<T>();
-    c.ndirty[0] = c.ndirty[1] = 0;
     c.sparse = 0;
     for (int j = 0; j < W; ++j) c.bitw[j] = c.cumw[j] = 0.f;
     a.ctrl[g] = c;
@@ -505,12 +497,6 @@ __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq
   }
 }
 
-template <typename T>
-__device__ __forceinline__ void flush_dirty(const BatchArgs<T> &a, int g, int level, uint32_t ndirty) {
-  ndirty = __reduce_add_sync(FULL, ndirty);
-  if ((threadIdx.x & 31) == 0 && ndirty) atomicAdd(&a.ctrl[g].ndirty[level & 1], ndirty);
-}
-
 // Top-down item: entries [i0, i1) of a TD queue class.  The frontier words and rows of
 // the entries are staged in shared memory, then an edge-balanced sweep (load-balanced
 // search on the degree prefix) ORs each frontier word into its unvisited neighbours
@@ -526,7 +512,7 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
   const T *vis = a.visited + (size_t)g * a.gstride;
   const uint32_t *q = queue_of(a, g, cls);
   const uint32_t qn = i1 - i0;
-  uint32_t insp = 0, writes = 0, ndirty = 0;
+  uint32_t insp = 0, writes = 0;
   for (uint32_t i = tid; i < qn; i += BLOCK) {
     const uint32_t v = queue_at(a, q, cls, i0 + i);
     const T f = wand(ldg(F + v), fmask);
@@ -556,12 +542,11 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       if (w[u] != 0xffffffffu) {
         insp++;
         const T b = filt ? wandn(fw[u], ldg(vis + w[u])) : fw[u];
-        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u], ndirty); }
+        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u]); }
       }
     }
   }
   flush_counts(sm, g, 0u, 0u, tid == 0 ? qn : 0u, insp, writes);
-  flush_dirty(a, g, level, ndirty);
 }
 
 // Bottom-up item: entries [i0, i1) of a BU queue class.
@@ -706,7 +691,7 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
   const T *vis = a.visited + (size_t)g * a.gstride;
   const T f = wand(ldg(F + c.v), fmask);
   if (wzero(f)) return;
-  uint32_t insp = 0, writes = 0, ndirty = 0;
+  uint32_t insp = 0, writes = 0;
   constexpr int U = 8;
   for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
     uint32_t w[U];
@@ -720,13 +705,12 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
       if (w[u] != 0xffffffffu) {
         insp++;
         const T b = filt ? wandn(f, ldg(vis + w[u])) : f;
-        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u], ndirty); }
+        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u]); }
       }
     }
   }
   const bool first = c.first && tid == 0;
   flush_counts(sm, g, 0u, 0u, first ? 1u : 0u, insp, writes);
-  flush_dirty(a, g, level, ndirty);
 }
 
 // Hub chunk, bottom-up: the CTA ORs a chunk of the hub's neighbours in waves, with a
@@ -930,7 +914,8 @@ constexpr int SAMPLE = SAMPLE_TILES * CVT;
 template <typename T>
 __device__ __forceinline__ bool commit_sparse(const BatchArgs<T> &a, const GroupCtrl<T> *c, int lc) {
   if (c->dir != 0) return false;
-  if ((unsigned long long)c->ndirty[lc & 1] * 4ull > (unsigned long long)a.nchunk32) return false;
+  // every write marks at most one chunk: the level's write count bounds the marked ones
+  if (a.lstat[(size_t)(c - a.ctrl) * MAXL + lc].writes * 4ull > (unsigned long long)a.nchunk32) return false;
   const uint32_t next = (uint32_t)lc + 1;
   switch (a.pol.mode) {
     case 0: case 1: return true;
@@ -956,23 +941,43 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
   uint32_t dg[CVT], rdg[CVT];  // out-degree (top-down rows), in-degree (bottom-up rows)
   bool live[CVT];              // chunk to read (dense commit, or marked dirty)
   uint8_t *dfl = a.dirty + (size_t)g * a.nchunk32;
+  uint8_t fl[CVT];
 #pragma unroll
   for (int k = 0; k < CVT; ++k) {
-    const size_t v = base + (size_t)k * BLOCK + tid;
+    const size_t ch = (base + (size_t)k * BLOCK + (size_t)(warp * 32)) >> 5;  // warp-uniform chunk
+    fl[k] = ch < a.nchunk32 ? dfl[ch] : (uint8_t)0;
     n[k] = wzero_value<T>();
     vv[k] = wzero_value<T>();
     dg[k] = rdg[k] = 0;
-    const size_t ch = (base + (size_t)k * BLOCK + (size_t)(warp * 32)) >> 5;  // warp-uniform chunk
-    const uint8_t fl = ch < a.nchunk32 ? dfl[ch] : (uint8_t)0;
-    if (fl && lane == 0) dfl[ch] = 0;  // consumed by this commit
-    live[k] = !sparse || fl;
-    if (v < nv && live[k]) {
-      n[k] = ld(N + v);
-      vv[k] = ld(vis + v);
-      dg[k] = __ldg(a.deg + v);
-      rdg[k] = a.directed ? __ldg(a.rdeg + v) : dg[k];
+  }
+  if (!sparse) {  // dense: the word loads do not wait for the chunk flags
+#pragma unroll
+    for (int k = 0; k < CVT; ++k) {
+      const size_t v = base + (size_t)k * BLOCK + tid;
+      live[k] = true;
+      if (v < nv) {
+        n[k] = ld(N + v);
+        vv[k] = ld(vis + v);
+        dg[k] = __ldg(a.deg + v);
+        rdg[k] = a.directed ? __ldg(a.rdeg + v) : dg[k];
+      }
+    }
+  } else {
+#pragma unroll
+    for (int k = 0; k < CVT; ++k) {
+      const size_t v = base + (size_t)k * BLOCK + tid;
+      live[k] = fl[k] != 0;
+      if (v < nv && live[k]) {
+        n[k] = ld(N + v);
+        vv[k] = ld(vis + v);
+        dg[k] = __ldg(a.deg + v);
+        rdg[k] = a.directed ? __ldg(a.rdeg + v) : dg[k];
+      }
     }
   }
+#pragma unroll
+  for (int k = 0; k < CVT; ++k)
+    if (fl[k] && lane == 0) dfl[(base + (size_t)k * BLOCK + (size_t)(warp * 32)) >> 5] = 0;  // consumed
   uint32_t bal[CVT][4];
   uint32_t wc[4] = {0, 0, 0, 0};
 #pragma unroll
@@ -1157,7 +1162,6 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->vpairs += np;
     c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
-    c->ndirty[lc & 1] = 0;
     c->sparse = sparse ? 1u : 0u;
     c->last_level = (uint32_t)lc;
     for (int k = 0; k < NQ; ++k) c->qlen[(lc + 1) & 1][k] = 0;  // target of commit lc+1

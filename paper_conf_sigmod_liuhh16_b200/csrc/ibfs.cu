@@ -977,7 +977,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   // groups per launch batch
   uint32_t G = o.groups_in_flight;
   if (G == 0) {
-    uint64_t want = (4ull << 20) / std::max<uint32_t>(nva, 1) + 1;
+    // auto: ~16 M status words per launch batch and at least 4 groups -- several groups
+    // share every level launch (a9), so one group's small levels overlap another's large
+    // ones and the host polls once per batch; the memory budget below caps it
+    uint64_t want = std::max<uint64_t>((16ull << 20) / std::max<uint32_t>(nva, 1) + 1, 4);
     G = (uint32_t)std::min<uint64_t>(want, MAX_G);
   }
   G = std::max<uint32_t>(1, std::min<uint32_t>({G, (uint32_t)MAX_G, n_groups}));
@@ -1127,7 +1130,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
       cudaEvent_t d0 = nullptr, d1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
-                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * 2 / Gb)));
+                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DEPTH_MINB / Gb)));
       const int first = flushed < 0 ? 1 : 0;
       depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
       launches++;

@@ -1310,7 +1310,13 @@ constexpr int DV = 128;               // columns per tile
 constexpr int DCW = 8;                // consumer warps
 constexpr int DTHREADS = DCW * 32;    // consumer threads
 constexpr int DSLOTS = 64;            // dense slots per round (DTHREADS / 4 parts)
-constexpr int DLB = 10;               // levels per pipeline stage
+#ifndef IBFS_DEPTH_DLB
+#define IBFS_DEPTH_DLB 10
+#endif
+#ifndef IBFS_DEPTH_MINB
+#define IBFS_DEPTH_MINB 2
+#endif
+constexpr int DLB = IBFS_DEPTH_DLB;   // levels per pipeline stage
 constexpr int DNS = 3;                // pipeline stages
 constexpr int DHDR = 32 + DV;         // stage header: k, run offset, c0, pad, nzbits[4]; slot -> column table
 
@@ -1417,7 +1423,7 @@ __device__ __forceinline__ uint32_t colb_off(uint32_t col, uint32_t ch) {
 // producer lanes arrived and its bytes landed (s_full[st], one expect_tx), "empty" when
 // every consumer warp has read it (s_empty[st]).
 template <typename T>
-__global__ void __launch_bounds__(DTHREADS + 32, 2)
+__global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
     depth_kernel(BatchArgs<T> a, int l0, int l1, int first) {
   using L = DepthLayout<T>;
   constexpr int W = WordBits<T>::value;

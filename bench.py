@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--alpha", type=float, default=4.0)
     ap.add_argument("--beta", type=float, default=24.0)
     ap.add_argument("--split-div", type=float, default=64.0)
+    ap.add_argument("--max-depth", type=int, default=0, help="k-hop mode (the 3-hop index of §8.7): 0 = plain BFS")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sources (0 = host cores)")
@@ -192,7 +193,7 @@ def main():
     out_dev = torch.empty((G * W, g.nv), dtype=torch.int8, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev) if args.config in ("c1", "c2", "c4") else None
     run_kw = dict(direction=args.direction, alpha=args.alpha, beta=args.beta, groups_in_flight=args.groups_in_flight,
-                  split_div=args.split_div)
+                  split_div=args.split_div, max_depth=(args.max_depth or None))
     stream = torch.cuda.current_stream(dev)
 
     def do_step(k, timing):
@@ -291,7 +292,7 @@ def main():
     # ---- CPU oracle beside it (rank 0, N = 1 only) -----------------------------------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(el, step_sources(0), args.cpu_sample)
+        cpu = cpu_baseline(el, step_sources(0), args.cpu_sample, args.max_depth or None)
 
     if rank == 0:
         line = {
@@ -299,11 +300,12 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(max_ms / args.steps, 3),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": f"u{W}",
             "data": "synthetic",
-            "config": {"workload": cfg.name, "generator": f"R-MAT/Kronecker (A,B,C)={cfg.abc}, seed {cfg.graph_seed}",
+            "config": {"workload": cfg.name + (f", {args.max_depth}-hop" if args.max_depth else ""), "generator": f"R-MAT/Kronecker (A,B,C)={cfg.abc}, seed {cfg.graph_seed}",
                        "scale": cfg.scale, "edgefactor": cfg.ef, "group_bits": W,
                        "sources_per_rank_per_step": G * W, "groups_per_rank_per_step": G,
                        "planner": "GroupBy", "direction": args.direction,
                        "groups_in_flight": args.groups_in_flight or "auto",
+                       "max_depth": args.max_depth or None,
                        "l2": ("flush 256 MiB between steps" if flush is not None
                               else "inputs > L2 (adjacency + per-group state), no flush"),
                        "parallelism": f"groups sharded over {world} rank(s), graph replicated"},
@@ -328,7 +330,7 @@ def main():
         dist.destroy_process_group()
 
 
-def cpu_baseline(el, sources, sample):
+def cpu_baseline(el, sources, sample, max_depth=None):
     """The oracle as it stands, timed on the host cores on a bounded sample."""
     import oracle
     cores = host_cores()
@@ -336,7 +338,7 @@ def cpu_baseline(el, sources, sample):
     s = np.asarray(sources[:k], dtype=np.uint32)
     og = oracle.OracleGraph.from_edges(el)  # adjacency build: setup, untimed
     t0 = time.perf_counter()
-    r = og.bfs(s, want_depths=False, threads=cores)
+    r = og.bfs(s, want_depths=False, threads=cores, max_depth=max_depth)
     dt = time.perf_counter() - t0
     return {"value": round(float(r.m_s.sum()) / dt / 1e9, 4), "unit": "GTEPS", "cores": min(cores, len(s)),
             "kind": "oracle", "seconds": round(dt, 2),

@@ -175,8 +175,17 @@ typedef struct {
      = k >= 1 stops every group after level k: vertices farther than k hops stay -1 and
      m_s counts the vertices within k hops.  0 = unbounded (plain BFS, the default). */
   uint32_t max_depth;
-  uint32_t reserved[3];
+  /* Traversal engine.  IBFS_ENGINE_BITWISE (default): the bitwise status words of §6
+      -- the product path.  IBFS_ENGINE_JOINT: the byte-per-instance Joint
+     Status Array of §4 (one warp per vertex builds the JFQ, the lanes of a
+     warp are the instances of a frontier), one group at a time with host-driven levels,
+     kept as the "Joint" rung of the ablation ladder (Fig. 15).  Same results
+     (max_depth included); split and groups_in_flight are bitwise-engine options. */
+  uint32_t engine;
+  uint32_t reserved[2];
 } ibfs_run_opts;
+
+enum { IBFS_ENGINE_BITWISE = 0, IBFS_ENGINE_JOINT = 1 };
 
 enum {
   IBFS_SPLIT_AUTO = 0,   /* small-frontier instances of a BU level run top-down */

@@ -38,7 +38,7 @@ class RunOpts(C.Structure):
                 ("schedule_len", C.c_uint32), ("alpha", C.c_float), ("beta", C.c_float),
                 ("groups_in_flight", C.c_uint32), ("cuda_stream", C.c_void_p), ("timing", C.c_uint32),
                 ("split", C.c_uint32), ("split_mod", C.c_uint32), ("split_div", C.c_float),
-                ("max_depth", C.c_uint32), ("reserved", C.c_uint32 * 3)]
+                ("max_depth", C.c_uint32), ("engine", C.c_uint32), ("reserved", C.c_uint32 * 2)]
 
 
 class LevelStats(C.Structure):

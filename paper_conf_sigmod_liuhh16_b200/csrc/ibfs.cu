@@ -27,6 +27,7 @@
 
 #include "../../include/ibfs.h"
 #include "kernels.cuh"
+#include "joint.cuh"
 #include "plan.h"
 
 using namespace ibfs;
@@ -1284,6 +1285,161 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   }
 }
 
+
+// ---- the byte-JSA joint engine (ablation rung "Joint", joint.cuh) ----------------------
+// One group at a time, host-driven levels (a JFQ scan, then the expand); the same
+// direction policy as the bitwise engine, decided on the host from the JFQ counters.
+void run_joint(const ibfs_graph *g, const uint32_t *sources, const uint32_t *csources, uint32_t n, uint32_t W,
+               int8_t *out_depths, const ibfs_run_opts &o, ibfs_stats *stats) {
+  using namespace joint;
+  cudaStream_t stream = (cudaStream_t)o.cuda_stream;
+  const uint32_t nv = g->nv, nva = g->nva;
+  const uint32_t n_groups = (n + W - 1) / W;
+  const bool out_dev = is_device_ptr(out_depths);
+  const bool out_host = out_depths && !out_dev;
+  Scratch sc(g->device, stream);
+  uint8_t *jsa = sc.get<uint8_t>((size_t)std::max<uint32_t>(nva, 1) * W);
+  uint32_t *jfq = sc.get<uint32_t>(std::max<uint32_t>(nva, 1));
+  unsigned long long *ctr = sc.get<unsigned long long>(4);
+  uint32_t *newcnt = sc.get<uint32_t>(W);
+  uint32_t *d_csrc = sc.get<uint32_t>(W);
+  unsigned long long *d_m = sc.get<unsigned long long>(W);
+  unsigned long long *d_dig = sc.get<unsigned long long>(W);
+  int8_t *staging = out_dev ? nullptr : sc.get<int8_t>((size_t)W * nv);
+  DevCache &dc = t_cache.get(g->device);
+  EventTimer timer(dc, true);
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win;
+  std::vector<ibfs_level_stats> per_level(MAXL);
+  ibfs_stats st{};
+  uint64_t launches = 0;
+  bool range_error = false;
+  const int grid = g->num_sms * 8;
+  JointArgs a{};
+  a.off = g->d_off;
+  a.adj = g->d_adj;
+  a.roff = g->directed ? g->d_roff : g->d_off;
+  a.radj = g->directed ? g->d_radj : g->d_adj;
+  a.deg = g->d_deg;
+  a.nva = nva;
+  a.W = (int)W;
+  a.jsa = jsa;
+  a.jfq = jfq;
+  a.ctr = ctr;
+  a.newcnt = newcnt;
+  std::vector<uint32_t> h_new(W);
+  std::vector<unsigned long long> h_m(W), h_dig(W);
+  for (uint32_t gi = 0; gi < n_groups; ++gi) {
+    const uint32_t rows = std::min<uint32_t>(W, n - gi * W);
+    int8_t *out = out_dev ? out_depths + (size_t)gi * W * nv : staging;
+    uint32_t act[4] = {0, 0, 0, 0};
+    for (uint32_t j = 0; j < rows; ++j)
+      if (csources[(size_t)gi * W + j] != NO_VERTEX) act[j >> 5] |= 1u << (j & 31);
+    cudaEvent_t w0 = timer.next(), w1 = timer.next();
+    CK(cudaEventRecord(w0, stream));
+    CK(cudaMemsetAsync(jsa, 0xff, (size_t)nva * W, stream));
+    CK(cudaMemcpyAsync(d_csrc, csources + (size_t)gi * W, rows * 4, cudaMemcpyHostToDevice, stream));
+    jsa_sources<<<1, W, 0, stream>>>(a, d_csrc, (int)rows);
+    launches++;
+    uint32_t dir = 0;  // direction of the level about to run: 0 TD, 1 BU
+    if (o.direction == IBFS_DIR_BU_FROM) dir = o.bu_from <= 1 ? 1 : 0;
+    if (o.direction == IBFS_DIR_SCHEDULE && o.schedule_len > 0) dir = (o.schedule[0] == 'B' || o.schedule[0] == 1);
+    for (int level = 1; level < MAXL; ++level) {
+      if ((act[0] | act[1] | act[2] | act[3]) == 0) break;
+      std::memcpy(a.act, act, sizeof(act));
+      unsigned long long h_ctr[4];
+      auto scan = [&](int bu) {
+        CK(cudaMemsetAsync(ctr, 0, 32, stream));
+        jfq_kernel<<<grid, 256, 0, stream>>>(a, level, bu);
+        launches++;
+        CK(cudaMemcpyAsync(h_ctr, ctr, 32, cudaMemcpyDeviceToHost, stream));
+        CK(cudaStreamSynchronize(stream));
+      };
+      const bool auto_now = o.direction == IBFS_DIR_AUTO ||
+                            (o.direction == IBFS_DIR_SCHEDULE && (uint32_t)level - 1 >= o.schedule_len);
+      if (level > 1 && auto_now) {
+        // reading #7 on the TD frontier of this level: TD -> BU when m_f * alpha > ne,
+        // BU -> TD when n_f * beta < nv_active
+        scan(0);
+        const double n_f = (double)h_ctr[0], m_f = (double)h_ctr[1];
+        dir = dir == 0 ? (m_f > 0 && m_f * o.alpha > (double)g->ne) : !(n_f * o.beta < (double)g->nv_active);
+        if (dir) scan(1);
+      } else {
+        if (o.direction == IBFS_DIR_TD_ONLY) dir = 0;
+        if (o.direction == IBFS_DIR_BU_FROM) dir = (uint32_t)level >= o.bu_from;
+        if (o.direction == IBFS_DIR_SCHEDULE && (uint32_t)level - 1 < o.schedule_len)
+          dir = (o.schedule[level - 1] == 'B' || o.schedule[level - 1] == 1);
+        scan((int)dir);
+      }
+      const uint32_t njfq = (uint32_t)h_ctr[0];
+      CK(cudaMemsetAsync(newcnt, 0, W * 4, stream));
+      if (njfq) {
+        joint_expand<<<grid, 256, 0, stream>>>(a, level, (int)dir, njfq);
+        launches++;
+      }
+      CK(cudaMemcpyAsync(h_new.data(), newcnt, W * 4, cudaMemcpyDeviceToHost, stream));
+      CK(cudaMemcpyAsync(h_ctr, ctr, 32, cudaMemcpyDeviceToHost, stream));
+      CK(cudaStreamSynchronize(stream));
+      uint64_t np = 0;
+      uint32_t nact[4] = {0, 0, 0, 0};
+      for (uint32_t j = 0; j < W; ++j)
+        if (h_new[j]) { np += h_new[j]; nact[j >> 5] |= 1u << (j & 31); }
+      ibfs_level_stats &P = per_level[level - 1];
+      if (dir) { P.bu_groups++; P.jfq_bu += njfq; st.levels_bu++; } else { P.td_groups++; P.jfq_td += njfq; st.levels_td++; }
+      P.inspected += h_ctr[2];
+      P.new_pairs += np;
+      st.edges_inspected += h_ctr[2];
+      st.max_levels = std::max<uint32_t>(st.max_levels, (uint32_t)level);
+      if (level >= 128 && np) range_error = true;
+      std::memcpy(act, nact, sizeof(act));
+      if (o.max_depth && (uint32_t)level >= o.max_depth) break;  // k-hop (§8.7)
+    }
+    // rows (vertex-major JSA -> instance-major int8), isolated sources, m_s
+    jsa_to_rows<<<grid, 256, 0, stream>>>(a, g->d_tbase, g->d_nzbits, nv, (int)rows, out);
+    launches++;
+    for (uint32_t j = 0; j < rows; ++j)
+      if (csources[(size_t)gi * W + j] == NO_VERTEX)
+        CK(cudaMemsetAsync(out + (size_t)j * nv + sources[(size_t)gi * W + j], 0, 1, stream));
+    CK(cudaMemsetAsync(d_m, 0, W * 8, stream));
+    jsa_ms<<<grid, W, 0, stream>>>(a, d_m);
+    launches++;
+    CK(cudaEventRecord(w1, stream));
+    win.push_back({w0, w1});
+    if (stats && stats->per_source_digest) {
+      BatchArgs<uint32_t> b{};
+      b.out = out;
+      b.nv = nv;
+      b.n_total = rows;
+      b.group0 = 0;
+      CK(cudaMemsetAsync(d_dig, 0, W * 8, stream));
+      digest_kernel<uint32_t><<<dim3(64, rows), BLOCK, 0, stream>>>(b, d_dig);
+      launches++;
+      CK(cudaMemcpyAsync(h_dig.data(), d_dig, W * 8, cudaMemcpyDeviceToHost, stream));
+    }
+    CK(cudaMemcpyAsync(h_m.data(), d_m, W * 8, cudaMemcpyDeviceToHost, stream));
+    if (out_host)
+      CK(cudaMemcpyAsync(out_depths + (size_t)gi * W * nv, staging, (size_t)rows * nv, cudaMemcpyDeviceToHost, stream));
+    CK(cudaStreamSynchronize(stream));
+    for (uint32_t r = 0; r < rows; ++r) {
+      st.edges_traversed += h_m[r];
+      if (stats && stats->per_source_m) stats->per_source_m[(size_t)gi * W + r] = h_m[r];
+      if (stats && stats->per_source_digest) stats->per_source_digest[(size_t)gi * W + r] = h_dig[r];
+    }
+  }
+  if (range_error) fail(IBFS_E_RANGE, "a depth exceeds 127 (int8 output)");
+  for (auto &p : win) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.traverse_ms += ms; }
+  st.n_groups = n_groups;
+  st.n_launches = launches;
+  if (stats) {
+    st.per_source_m = stats->per_source_m;
+    st.per_source_digest = stats->per_source_digest;
+    st.level_cap = stats->level_cap;
+    st.per_level = stats->per_level;
+    if (st.per_level)
+      for (uint32_t i = 0; i < st.level_cap; ++i) st.per_level[i] = i < (uint32_t)MAXL ? per_level[i] : ibfs_level_stats{};
+    *stats = st;
+  }
+}
+
 }  // namespace
 
 extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_t n, uint32_t group_bits,
@@ -1298,6 +1454,7 @@ extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_
     if (o.direction == IBFS_DIR_SCHEDULE && o.schedule_len > 0 && !o.schedule) fail(IBFS_E_INVALID, "schedule is NULL");
     if (!(o.alpha > 0) || !(o.beta > 0)) fail(IBFS_E_INVALID, "alpha and beta must be > 0");
     if (o.split > IBFS_SPLIT_FORCE) fail(IBFS_E_INVALID, "bad split mode");
+    if (o.engine > IBFS_ENGINE_JOINT) fail(IBFS_E_INVALID, "bad engine");
     if (o.split == IBFS_SPLIT_FORCE && o.split_mod == 0) fail(IBFS_E_INVALID, "split_mod must be > 0");
     if (o.split == IBFS_SPLIT_AUTO && !(o.split_div > 0)) fail(IBFS_E_INVALID, "split_div must be > 0");
     if (stats) {
@@ -1323,7 +1480,8 @@ extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_
     for (uint32_t r = 0; r < n; ++r)
       if (hs[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
     for (uint32_t r = 0; r < n; ++r) hcs[r] = host_compact_id(g, hs[r]);
-    if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
+    if (o.engine == IBFS_ENGINE_JOINT) run_joint(g, hs.data(), hcs.data(), n, group_bits, out_depths, o, stats);
+    else if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
     else if (group_bits == 64) run_typed<unsigned long long>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
     else run_typed<u128>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
   });

@@ -206,9 +206,12 @@ class Graph:
             schedule: str | None = None, bu_from: int = 2, alpha: float = 4.0, beta: float = 24.0,
             groups_in_flight: int = 0, stream=None, timing: bool = False, want_m: bool = True,
             want_digest: bool = False, level_cap: int = 130, split: str = "auto",
-            split_mod: int = 2, split_div: float = 64.0, max_depth: int | None = None):
+            split_mod: int = 2, split_div: float = 64.0, max_depth: int | None = None,
+            engine: str = "bitwise"):
         """n concurrent BFS instances; returns (depths, RunStats).
 
+        engine: "bitwise" (the product path) or "joint" (the byte-JSA joint traversal of §4,
+        kept for the ablation ladder; same results).
         max_depth = k >= 1: k-hop mode, the first k levels only (the reachability index of
         §8.7); vertices farther than k hops are -1.  None = plain BFS.
 
@@ -261,6 +264,7 @@ class Graph:
             if int(max_depth) < 1:
                 raise ValueError("max_depth must be >= 1 (None = unbounded)")
             opts.max_depth = int(max_depth)
+        opts.engine = {"bitwise": 0, "joint": 1}[engine]
         st = _lib.Stats()
         m_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_m else None
         d_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_digest else None

@@ -464,3 +464,56 @@ def test_directed_from_csr_matches_from_edges_and_khop():
     bad_off[1:-1] = np.minimum(bad_off[1:-1] + 1, bad_off[-1])
     with pytest.raises(Exception):
         P.Graph.from_csr(off, adj, rev_offsets=bad_off, rev_adj=radj)
+
+
+# ------------------------------------- byte-JSA joint engine (ablation rung, NEXT #3)
+# §4: the Joint Status Array keeps a depth byte per (vertex, instance); the
+# same depths, m_s and digests as the oracle (and as the bitwise engine).
+@pytest.mark.parametrize("W", [32, 64, 128])
+@pytest.mark.parametrize("kind", SCHEDULES)
+def test_joint_engine_fig1(W, kind):
+    fx = read_fig1()
+    el = ibfs_gen.from_pairs(fx["nv"], fx["edges"])
+    g = P.Graph.from_edgelist(el)
+    d, st = gpu_depths(g, fx["sources"], W, engine="joint", want_digest=True, **run_kwargs(kind))
+    np.testing.assert_array_equal(d, fx["depths"])
+    ref = oracle.bfs(el, fx["sources"])
+    np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+    np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+
+
+def test_joint_engine_random_tiny():
+    rng = np.random.default_rng(909)
+    for trial in range(60):
+        nv = int(rng.integers(1, 60))
+        m = int(rng.integers(0, 3 * nv + 1))
+        pairs = [(int(rng.integers(nv)), int(rng.integers(nv))) for _ in range(m)]
+        directed = bool(trial % 3 == 0)
+        el = ibfs_gen.from_pairs(nv, pairs if pairs else np.zeros((0, 2)), directed=directed)
+        n = int(rng.integers(1, 200))
+        src = rng.integers(0, nv, size=n).astype(np.uint32)
+        W = int(rng.choice([32, 64, 128]))
+        kind = SCHEDULES[trial % len(SCHEDULES)]
+        k = int(rng.integers(1, 4)) if trial % 5 == 0 else None
+        g = P.Graph.from_edgelist(el)
+        d, st = gpu_depths(g, src, W, engine="joint", want_digest=True, max_depth=k, **run_kwargs(kind, rng))
+        ref = oracle.bfs(el, src, max_depth=k)
+        np.testing.assert_array_equal(d, ref.depths, err_msg=f"trial {trial} W={W} {kind} dir={directed} k={k}")
+        np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+        np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+
+
+@pytest.mark.parametrize("name", ["c1", "c2", "d2"])
+def test_joint_engine_configs(name):
+    cfg = ibfs_gen.CONFIGS[name]
+    el = cfg.edges()
+    src = cfg.sources(el)
+    g = P.Graph.from_edgelist(el)
+    s = src[g.plan(src, cfg.group_bits)]
+    d, st = gpu_depths(g, s, cfg.group_bits, engine="joint", want_digest=True)
+    db, stb = gpu_depths(g, s, cfg.group_bits, want_digest=True)
+    np.testing.assert_array_equal(d, db)  # bitwise and joint engines agree
+    ref = oracle.bfs(el, s)
+    np.testing.assert_array_equal(d, ref.depths)
+    np.testing.assert_array_equal(st.per_source_m, ref.m_s)
+    np.testing.assert_array_equal(st.per_source_digest, ref.digest)

@@ -2,8 +2,10 @@
 Fig. 20): the same sources traversed
   (1) sequentially -- one BFS instance per call (W = 32 word, one active bit), the
       "sequential concurrent BFS" of P:L217 on this library's kernels;
-  (2) bitwise joint traversal, random grouping (plan mode "random");
-  (3) bitwise joint traversal + outdegree-based GroupBy (§5.2).
+  (2) joint traversal with the byte-per-instance Joint Status Array (§4, engine "joint"),
+      random grouping;
+  (3) bitwise joint traversal, random grouping (plan mode "random");
+  (4) bitwise joint traversal + outdegree-based GroupBy (§5.2).
 GTEPS = sum of m_s / device time (CUDA events).  usage: ablation.py [config] [n_sources]"""
 import os
 import sys
@@ -48,18 +50,19 @@ def sequential():
     return e
 
 
-def joint(mode):
+def joint(mode, engine="bitwise"):
     perm = g.plan(src, W, mode=mode)
     s = src[perm]
 
     def f():
-        _, st = g.run(s, W, out=out[: len(s)], stream=stream)
+        _, st = g.run(s, W, out=out[: len(s)], stream=stream, engine=engine)
         return st.edges_traversed
     return f
 
 
 res = {"config": cfg.name, "sources": int(len(src)),
        "sequential (1 instance per call, 64-source sample)": timed(sequential),
+       "joint byte-JSA (§4), random grouping": timed(joint("random", "joint")),
        "bitwise, random grouping": timed(joint("random")),
        "bitwise + GroupBy": timed(joint("groupby"))}
 print(json.dumps(res, indent=1))

@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--max-depth", type=int, default=0, help="k-hop mode (the 3-hop index of §8.7): 0 = plain BFS")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-clocks", action="store_true", help="diagnostics: no nvidia-smi sampling")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sources (0 = host cores)")
     ap.add_argument("--json-out", default="")
     return ap.parse_args()
@@ -208,7 +209,8 @@ def main():
     if world > 1:
         dist.barrier()
     sampler = ClockSampler(local)
-    sampler.start()
+    if not args.no_clocks:
+        sampler.start()
     time.sleep(0.25)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()

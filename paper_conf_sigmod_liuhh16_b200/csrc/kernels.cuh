@@ -1311,10 +1311,10 @@ constexpr int DCW = 8;                // consumer warps
 constexpr int DTHREADS = DCW * 32;    // consumer threads
 constexpr int DSLOTS = 64;            // dense slots per round (DTHREADS / 4 parts)
 #ifndef IBFS_DEPTH_DLB
-#define IBFS_DEPTH_DLB 10
+#define IBFS_DEPTH_DLB 5
 #endif
 #ifndef IBFS_DEPTH_MINB
-#define IBFS_DEPTH_MINB 2
+#define IBFS_DEPTH_MINB 3
 #endif
 constexpr int DLB = IBFS_DEPTH_DLB;   // levels per pipeline stage
 constexpr int DNS = 3;                // pipeline stages

@@ -200,6 +200,7 @@ struct ibfs_graph {
   std::vector<uint64_t> h_roff;
   std::vector<uint32_t> h_tbase, h_nzbits;
   int num_sms = 148;
+  size_t total_mem = 0;  // device memory (bytes), queried once at load
   int level_blocks_per_sm[3] = {1, 1, 1};  // co-resident level_kernel CTAs per SM (W = 32, 64, 128)
 };
 
@@ -438,6 +439,10 @@ void finish_graph(ibfs_graph *g) {
   }
   int dev = g->device;
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, dev));
+  {
+    size_t free_b = 0;
+    CK(cudaMemGetInfo(&free_b, &g->total_mem));
+  }
   CK(cudaFuncSetAttribute(level_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)sizeof(TileQueue<uint32_t>)));
   CK(cudaFuncSetAttribute(level_kernel<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -923,7 +928,7 @@ extern "C" void ibfs_run_opts_default(ibfs_run_opts *o) {
 
 namespace {
 
-constexpr int LEVELS_PER_CHECK = 2;
+constexpr int LEVELS_PER_CHECK = 4;  // levels per polled chunk; two chunks stay queued ahead
 
 // Per-thread, per-device cache of CUDA events and a pinned host word buffer: creating
 // them per call (cudaEventCreate, cudaMallocHost) costs far more than a small level.
@@ -987,8 +992,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   G = std::max<uint32_t>(1, std::min<uint32_t>({G, (uint32_t)MAX_G, n_groups}));
   const size_t gstride = ((size_t)nva + 16) & ~(size_t)15;
   const size_t rows_bytes_per_group = (size_t)W * nv;
-  size_t free_b = 0, total_b = 0;
-  CK(cudaMemGetInfo(&free_b, &total_b));
+  const size_t total_b = g->total_mem;
   // memory: visited + R snapshot slots per group (+ device rows if the caller's buffer
   // is not on the device); R >= 4, up to one slot per level when memory allows
   auto need = [&](uint32_t gg, uint32_t r) {
@@ -996,7 +1000,6 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   };
   // The budget depends on the device size only (not on the momentary free memory), so
   // repeated calls request identical scratch and the stream-ordered pool reuses it.
-  (void)free_b;
   const size_t budget = total_b / 100 * 35;
   while (G > 1 && need(G, 4) > budget) G = (G + 1) / 2;
   uint32_t R = 4;

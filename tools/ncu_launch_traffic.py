@@ -1,0 +1,57 @@
+"""Per-kernel summary of an ncu metrics CSV (one row per launch x metric): launches, time,
+share, and DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum).
+usage: ncu_launch_traffic.py <csv> [config kernel-regex=name ... --json profiles/ncu_traffic.json]
+With --json, writes the mean DRAM bytes per launch of each named kernel into the traffic
+file bench.py reads (same launch set as bench's `achieved`: every launch of the step)."""
+import csv
+import json
+import re
+import sys
+from collections import defaultdict
+
+path = sys.argv[1]
+rows = [r for r in csv.reader(open(path)) if r]
+h = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
+hdr = rows[h]
+I = {k: hdr.index(k) for k in ("ID", "Kernel Name", "Metric Name", "Metric Unit", "Metric Value")}
+launch = defaultdict(dict)
+names = {}
+for r in rows[h + 1:]:
+    if len(r) < len(hdr):
+        continue
+    lid = int(r[I["ID"]])
+    names[lid] = r[I["Kernel Name"]].split("(")[0].replace("void ", "")
+    v = float(r[I["Metric Value"]].replace(",", ""))
+    u = r[I["Metric Unit"]]
+    scale = {"ns": 1e-6, "nsecond": 1e-6, "us": 1e-3, "usecond": 1e-3, "ms": 1.0, "msecond": 1.0,
+             "byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}.get(u, 1.0)
+    launch[lid][r[I["Metric Name"]]] = v * scale
+agg = defaultdict(lambda: [0, 0.0, 0.0])
+for lid, m in launch.items():
+    a = agg[names[lid]]
+    a[0] += 1
+    a[1] += m.get("gpu__time_duration.sum", 0.0)
+    a[2] += m.get("dram__bytes_read.sum", 0.0) + m.get("dram__bytes_write.sum", 0.0)
+tot = sum(a[1] for a in agg.values()) or 1.0
+print("| kernel | launches | total ms | ms/launch | share | DRAM MB/launch | DRAM GB/s |")
+print("|---|---|---|---|---|---|---|")
+for k, (n, t, b) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
+    print(f"| `{k}` | {n} | {t:.3f} | {t / n:.4f} | {100 * t / tot:.1f}% | {b / n / 1e6:.1f} | {b / (t * 1e-3) / 1e9 if t else 0:.0f} |")
+if "--json" in sys.argv:
+    i = sys.argv.index("--json")
+    out = sys.argv[i + 1]
+    config = sys.argv[2]
+    try:
+        j = json.load(open(out))
+    except Exception:
+        j = {}
+    for spec in sys.argv[3:i]:
+        rx, name = spec.split("=")
+        sel = [(n, t, b) for k, (n, t, b) in agg.items() if re.search(rx, k)]
+        n = sum(x[0] for x in sel)
+        b = sum(x[2] for x in sel)
+        j.setdefault(config, {})[name] = {
+            "dram_bytes_per_launch": b / n if n else None, "launches": n, "source": path.split("/")[-1],
+            "note": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none, "
+                    "every launch of one bench step (the launch set bench.py's achieved averages over)"}
+    json.dump(j, open(out, "w"), indent=1)

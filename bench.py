@@ -313,6 +313,11 @@ def main():
                        "parallelism": f"groups sharded over {world} rank(s), graph replicated"},
             "traverse_gteps": round(edges / (traverse_ms * 1e-3) / 1e9, 2) if traverse_ms else None,
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "timeline": {"timed_ms": round(max_ms, 3), "traverse_ms": round(traverse_ms, 3),
+                         "level_gap_ms": round(sum(s.level_gap_ms for s in sts), 3),
+                         "note": "traverse = device windows of the ibfs_run_ex calls; level_gap = device idle "
+                                 "between consecutive level kernels (in-kernel globaltimer); the rest of "
+                                 "timed_ms is between calls / batches"},
             "gpu_launches": int(sum(s.n_launches for s in sts)),
             "clocks": clocks,
             "setup": {"gen_s": round(gen_s, 2), "load_s": round(load_s, 2), "plan_ms": round(plan_ms, 2),

@@ -223,6 +223,8 @@ typedef struct {
   double level_ms, expand_ms, commit_ms, init_ms, depth_ms;
   uint64_t level_launches, init_launches, depth_launches;
   uint64_t expand_bytes, commit_bytes, init_bytes, depth_bytes;
+  double level_gap_ms;  /* device idle between consecutive level kernels of a batch (in-kernel
+                           globaltimer stamps): launch latency plus any host polling stall */
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */
   uint64_t *per_source_digest;  /* [n] sum over reached v of splitmix64((v<<8)|(d+1)) */

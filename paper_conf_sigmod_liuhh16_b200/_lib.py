@@ -60,7 +60,7 @@ class Stats(C.Structure):
                 ("init_ms", C.c_double), ("depth_ms", C.c_double),
                 ("level_launches", C.c_uint64), ("init_launches", C.c_uint64), ("depth_launches", C.c_uint64),
                 ("expand_bytes", C.c_uint64), ("commit_bytes", C.c_uint64), ("init_bytes", C.c_uint64),
-                ("depth_bytes", C.c_uint64),
+                ("depth_bytes", C.c_uint64), ("level_gap_ms", C.c_double),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),
                 ("level_cap", C.c_uint32), ("per_level", C.c_void_p)]
 

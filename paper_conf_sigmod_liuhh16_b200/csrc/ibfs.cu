@@ -1266,6 +1266,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         per_level[l - 2].commit_ms += cms;
       }
     }
+    for (int l = 1; l + 1 < MAXL; ++l) {  // idle between level l's last CTA and level l+1's first
+      const unsigned long long e = h_ts[(size_t)l * 3 + 2], b = h_ts[(size_t)(l + 1) * 3];
+      if (e && b != ~0ull && b > e) st.level_gap_ms += (b - e) * 1e-6;
+    }
   }
   if (range_error) fail(IBFS_E_RANGE, "a depth exceeds 127 (int8 output)");
   // times

@@ -88,6 +88,7 @@ class RunStats:
     commit_bytes: int
     init_bytes: int
     depth_bytes: int
+    level_gap_ms: float
     per_source_m: np.ndarray | None = None
     per_source_digest: np.ndarray | None = None
     per_level: list = field(default_factory=list)

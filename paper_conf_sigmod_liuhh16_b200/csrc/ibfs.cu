@@ -983,10 +983,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   // groups per launch batch
   uint32_t G = o.groups_in_flight;
   if (G == 0) {
-    // auto: ~16 M status words per launch batch and at least 4 groups -- several groups
+    // auto: ~32 M status words per launch batch and at least 4 groups -- several groups
     // share every level launch (a9), so one group's small levels overlap another's large
     // ones and the host polls once per batch; the memory budget below caps it
-    uint64_t want = std::max<uint64_t>((16ull << 20) / std::max<uint32_t>(nva, 1) + 1, 4);
+    uint64_t want = std::max<uint64_t>((32ull << 20) / std::max<uint32_t>(nva, 1) + 1, 4);
     G = (uint32_t)std::min<uint64_t>(want, MAX_G);
   }
   G = std::max<uint32_t>(1, std::min<uint32_t>({G, (uint32_t)MAX_G, n_groups}));

@@ -45,7 +45,7 @@ constexpr int LIGHT_DEG = 32;    // degree <= LIGHT_DEG: light
 constexpr int HUB_T = 8192;      // degree > HUB_T: hub (chunked rows)
 constexpr int CHUNK = 8192;      // hub-row edges per work item
 constexpr int MAXL = 130;        // level index 1..129 (129 only detects depth > 127)
-constexpr int MAX_G = 64;        // groups per launch batch
+constexpr int MAX_G = 128;       // groups per launch batch
 constexpr unsigned FULL = 0xffffffffu;
 #ifndef IBFS_EXPAND_MINB
 #define IBFS_EXPAND_MINB 3  // min resident expand CTAs per SM (register cap)
@@ -791,10 +791,19 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     sm.pre[i] = n;
   }
   __syncthreads();
-  if (tid == 0) {  // exclusive prefix (<= 384 slots)
-    uint32_t run = 0;
-    for (int i = 0; i < nslot; ++i) { const uint32_t x = sm.pre[i]; sm.pre[i] = run; run += x; }
-    sm.pre[nslot] = run;
+  if (tid < 32) {  // exclusive prefix over the <= 6 * MAX_G slots: lane-contiguous segments
+    const int seg = (nslot + 31) / 32, i0 = min(tid * seg, nslot), i1 = min(i0 + seg, nslot);
+    uint32_t sum = 0;
+    for (int i = i0; i < i1; ++i) sum += sm.pre[i];
+    uint32_t inc = sum;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, inc, d);
+      if (tid >= d) inc += y;
+    }
+    uint32_t run = inc - sum;
+    for (int i = i0; i < i1; ++i) { const uint32_t x = sm.pre[i]; sm.pre[i] = run; run += x; }
+    if (tid == 31) sm.pre[nslot] = inc;
   }
   __syncthreads();
   const uint32_t total = sm.pre[nslot];

@@ -52,6 +52,6 @@ if "--json" in sys.argv:
         b = sum(x[2] for x in sel)
         j.setdefault(config, {})[name] = {
             "dram_bytes_per_launch": b / n if n else None, "launches": n, "source": path.split("/")[-1],
-            "note": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none, "
-                    "every launch of one bench step (the launch set bench.py's achieved averages over)"}
+            "note": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none over a bench.py run: "
+                    "every launch of the run (the launch set bench.py achieved averages over)"}
     json.dump(j, open(out, "w"), indent=1)

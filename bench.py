@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--alpha", type=float, default=4.0)
     ap.add_argument("--beta", type=float, default=24.0)
     ap.add_argument("--split-div", type=float, default=64.0)
+    ap.add_argument("--plan-hops", type=int, default=1, help="GroupBy hub radius (1 = the paper's steps, 2 = 2-hop anchors)")
     ap.add_argument("--max-depth", type=int, default=0, help="k-hop mode (the 3-hop index of §8.7): 0 = plain BFS")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -144,10 +145,10 @@ def ncu_traffic(config: str, kernel: str):
         return None, None
 
 
-def plan_for(cfg, g, el, W):
+def plan_for(cfg, g, el, W, hops=1):
     src = cfg.sources(el)
     t0 = time.perf_counter()
-    perm = g.plan(src, W)
+    perm = g.plan(src, W, hops=hops)
     plan_ms = (time.perf_counter() - t0) * 1e3
     return src[perm], plan_ms
 
@@ -177,7 +178,7 @@ def main():
     t0 = time.perf_counter()
     g = P.Graph.from_edgelist(el, device=local)
     load_s = time.perf_counter() - t0
-    s_plan, plan_ms = plan_for(cfg, g, el, W)
+    s_plan, plan_ms = plan_for(cfg, g, el, W, args.plan_hops)
     n = len(s_plan)
     n_groups = (n + W - 1) // W
     deg = np.diff(g.export_csr()[0]).astype(np.int64) if cfg.scale <= 24 else None
@@ -305,7 +306,7 @@ def main():
             "config": {"workload": cfg.name + (f", {args.max_depth}-hop" if args.max_depth else ""), "generator": f"R-MAT/Kronecker (A,B,C)={cfg.abc}, seed {cfg.graph_seed}",
                        "scale": cfg.scale, "edgefactor": cfg.ef, "group_bits": W,
                        "sources_per_rank_per_step": G * W, "groups_per_rank_per_step": G,
-                       "planner": "GroupBy", "direction": args.direction,
+                       "planner": "GroupBy" + (f" (hops={args.plan_hops})" if args.plan_hops != 1 else ""), "direction": args.direction,
                        "groups_in_flight": args.groups_in_flight or "auto",
                        "max_depth": args.max_depth or None,
                        "l2": ("flush 256 MiB between steps" if flush is not None

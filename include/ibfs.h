@@ -109,7 +109,10 @@ typedef struct {
   uint32_t q;        /* hub: outdegree > q (default 128) */
   uint32_t n_p;      /* number of Rule-1 bounds in p[] (1..8; default 4) */
   uint32_t p[8];     /* ascending Rule-1 bounds (default 4, 16, 64, 128) */
-  uint32_t hops;     /* hub search radius; only 1 is implemented (default 1) */
+  uint32_t hops;     /* 1 (default): the steps above.  2: "not required ... directly ... as long
+                        as within the first several levels" -- the bucket leftovers and
+                        the Rule-1 rejects that have a hub are ordered by their 2-hop anchor
+                        (the larger of hub(r) and hub(hub(r)) by degree) before grouping */
   uint64_t seed;     /* seeded Fisher-Yates for the random remainder / random mode (3) */
 } ibfs_plan_params;
 

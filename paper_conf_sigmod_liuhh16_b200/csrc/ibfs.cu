@@ -881,7 +881,7 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
     if (params) pp = *params; else ibfs_plan_params_default(&pp);
     if (pp.mode > 2) fail(IBFS_E_INVALID, "plan mode must be 0, 1 or 2");
     if (pp.mode == 0 && (pp.n_p < 1 || pp.n_p > 8)) fail(IBFS_E_INVALID, "n_p must be 1..8");
-    if (pp.mode == 0 && pp.hops != 1) fail(IBFS_E_UNSUPPORTED, "only hops = 1 is implemented");
+    if (pp.mode == 0 && pp.hops != 1 && pp.hops != 2) fail(IBFS_E_INVALID, "hops must be 1 or 2");
     if (out_n_groups) *out_n_groups = (n + group_bits - 1) / group_bits;
     if (n == 0) return;
     std::vector<uint32_t> hsrc(n);
@@ -890,7 +890,7 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
     for (uint32_t r = 0; r < n; ++r)
       if (hsrc[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
     for (uint32_t r = 0; r < n; ++r) hsrc[r] = host_compact_id(g, hsrc[r]);  // planner works on compacted ids
-    std::vector<uint32_t> hub(n, 0xffffffffu), sdeg(n, 0);
+    std::vector<uint32_t> hub(n, 0xffffffffu), sdeg(n, 0), anchor;
     if (pp.mode == 0) {
       uint32_t *d_src = nullptr, *d_hub = nullptr, *d_sdeg = nullptr;
       CK(cudaMalloc(&d_src, (size_t)n * 4));
@@ -903,13 +903,36 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
       cudaError_t e = cudaGetLastError();
       if (e == cudaSuccess) e = cudaMemcpy(hub.data(), d_hub, (size_t)n * 4, cudaMemcpyDeviceToHost);
       if (e == cudaSuccess) e = cudaMemcpy(sdeg.data(), d_sdeg, (size_t)n * 4, cudaMemcpyDeviceToHost);
+      if (e == cudaSuccess && pp.hops == 2) {
+        // hub of each source's hub (the same search from the hub vertex); anchor = the
+        // larger of the two by (degree desc, id asc)
+        std::vector<uint32_t> hv(n), hub2(n, 0xffffffffu);
+        for (uint32_t r = 0; r < n; ++r) hv[r] = hub[r] == 0xffffffffu ? NO_VERTEX : hub[r];
+        e = cudaMemcpy(d_src, hv.data(), (size_t)n * 4, cudaMemcpyHostToDevice);
+        if (e == cudaSuccess) {
+          hub_kernel<<<blocks, 256>>>(g->d_off, g->d_adj, g->d_deg, d_src, n, pp.q, uniform, d_hub, d_sdeg);
+          e = cudaGetLastError();
+        }
+        if (e == cudaSuccess) e = cudaMemcpy(hub2.data(), d_hub, (size_t)n * 4, cudaMemcpyDeviceToHost);
+        anchor.assign(n, 0xffffffffu);
+        for (uint32_t r = 0; r < n; ++r) {
+          uint32_t a = hub[r];
+          const uint32_t b = hub2[r];
+          if (a != 0xffffffffu && b != 0xffffffffu) {
+            const uint64_t da = g->h_off[a + 1] - g->h_off[a], db = g->h_off[b + 1] - g->h_off[b];
+            if (db > da || (db == da && b < a)) a = b;
+          }
+          anchor[r] = a;
+        }
+      }
       cudaFree(d_src);
       cudaFree(d_hub);
       cudaFree(d_sdeg);
       CK(e);
     }
     auto deg_of = [&](uint32_t x) -> uint64_t { return g->h_off[x + 1] - g->h_off[x]; };
-    ibfs::plan::make_plan(pp, group_bits, n, hub, sdeg, deg_of, out_perm);
+    ibfs::plan::make_plan(pp, group_bits, n, hub, sdeg, deg_of, out_perm,
+                          pp.mode == 0 && pp.hops == 2 ? &anchor : nullptr);
   });
 }
 

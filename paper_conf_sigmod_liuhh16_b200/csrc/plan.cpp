@@ -10,7 +10,7 @@
 // order, emit full W-groups per bucket (buckets visited by hub degree desc, id asc),
 // then concatenate the bucket leftovers in the same order, then degree-0 sources, then a
 // seeded shuffle of the remaining sources.  hub(r) is computed on the device
-// (hub_kernel in ibfs.cu).
+// (hub_kernel in ibfs.cu).  hops = 2 orders the leftovers by their 2-hop anchor (below).
 #include "plan.h"
 
 #include <algorithm>
@@ -35,7 +35,8 @@ void seeded_shuffle(std::vector<uint32_t> &items, uint64_t seed) {
 
 void make_plan(const ibfs_plan_params &pp, uint32_t group_bits, uint32_t n,
                const std::vector<uint32_t> &hub, const std::vector<uint32_t> &sdeg,
-               const std::function<uint64_t(uint32_t)> &deg_of, uint32_t *out_perm) {
+               const std::function<uint64_t(uint32_t)> &deg_of, uint32_t *out_perm,
+               const std::vector<uint32_t> *anchor) {
   std::vector<uint32_t> perm;
   perm.reserve(n);
   if (pp.mode == 2) {
@@ -74,15 +75,39 @@ void make_plan(const ibfs_plan_params &pp, uint32_t group_bits, uint32_t n,
         }
       }
     }
-    for (uint32_t h : order) {
-      Bucket &b = buckets[h];
-      perm.insert(perm.end(), b.items.begin() + b.head, b.items.end());
+    if (!anchor) {
+      for (uint32_t h : order) {
+        Bucket &b = buckets[h];
+        perm.insert(perm.end(), b.items.begin() + b.head, b.items.end());
+      }
     }
-    std::vector<uint32_t> other;
+    std::vector<uint32_t> other, late;
     for (uint32_t r = 0; r < n; ++r) {
       if (bucketed[r]) continue;
       if (sdeg[r] == 0) perm.push_back(r);
+      else if (anchor && hub[r] != NO_HUB) late.push_back(r);
       else other.push_back(r);
+    }
+    if (anchor) {
+      // hops = 2 ("as long as within the first several levels"): the bucket
+      // leftovers, and the sources Rule 1 never admitted that still have a hub, ordered
+      // by their 2-hop anchor (the larger of hub(r) and hub(hub(r)): the core vertex they
+      // reach within two levels), then by hub, then by position
+      std::vector<uint32_t> rest;
+      for (uint32_t h : order) {
+        Bucket &b = buckets[h];
+        rest.insert(rest.end(), b.items.begin() + b.head, b.items.end());
+      }
+      rest.insert(rest.end(), late.begin(), late.end());
+      std::vector<uint32_t> pos(n, 0);
+      for (uint32_t i = 0; i < rest.size(); ++i) pos[rest[i]] = i;
+      std::stable_sort(rest.begin(), rest.end(), [&](uint32_t x, uint32_t y) {
+        const uint32_t ax = (*anchor)[x], ay = (*anchor)[y];
+        if (ax != ay) return by_degree(ax, ay);
+        if (hub[x] != hub[y]) return by_degree(hub[x], hub[y]);
+        return pos[x] < pos[y];
+      });
+      perm.insert(perm.end(), rest.begin(), rest.end());
     }
     seeded_shuffle(other, pp.seed);
     perm.insert(perm.end(), other.begin(), other.end());

@@ -244,6 +244,7 @@ def test_planner_matches_oracle_planner(W):
         og = oracle.OracleGraph.from_edges(el)
         off, adj = og.adjacency()
         np.testing.assert_array_equal(g.plan(src, W), planner.groupby(off, adj, src, W))
+        np.testing.assert_array_equal(g.plan(src, W, hops=2), planner.groupby(off, adj, src, W, hops=2))
         np.testing.assert_array_equal(g.plan(src, W, mode="random", seed=9), planner.random_plan(len(src), 9))
         np.testing.assert_array_equal(g.plan(src, W, mode="identity"), np.arange(len(src)))
     el = ibfs_gen.rmat(12, 16, ibfs_gen.KRONECKER, seed=1)
@@ -251,6 +252,7 @@ def test_planner_matches_oracle_planner(W):
     g = P.Graph.from_edgelist(el)
     off, adj = oracle.OracleGraph.from_edges(el).adjacency()
     np.testing.assert_array_equal(g.plan(allv, W), planner.groupby(off, adj, allv, W))
+    np.testing.assert_array_equal(g.plan(allv, W, hops=2), planner.groupby(off, adj, allv, W, hops=2))
 
 
 def test_csr_build_matches_oracle_adjacency():

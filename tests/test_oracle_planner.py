@@ -74,3 +74,33 @@ def test_groupby_raises_sharing_on_apsp_pool():
     sd_g = mean_sd(planner.groupby(off, adj, src, W))
     sd_r = mean_sd(planner.random_plan(len(src), 3))
     assert sd_g > 1.2 * sd_r
+
+
+def test_groupby_hops2_invariants_and_anchor_order():
+    """hops = 2: a permutation, deterministic, full 1-hop groups first, and the
+    remaining hubbed sources contiguous per 2-hop anchor."""
+    el = ibfs_gen.rmat(12, 16, ibfs_gen.KRONECKER, seed=5)
+    og = oracle.OracleGraph.from_edges(el)
+    off, adj = og.adjacency()
+    src = ibfs_gen.sample_sources(el, 1024, 7)
+    p1 = planner.groupby(off, adj, src, 32)
+    p2 = planner.groupby(off, adj, src, 32, hops=2)
+    assert sorted(p2.tolist()) == list(range(len(src)))
+    np.testing.assert_array_equal(p2, planner.groupby(off, adj, src, 32, hops=2))
+    hub, sdeg = planner.hubs(off, adj, src, 128)
+    deg = np.diff(off.astype(np.int64))
+    # the full groups of step 3 are identical in both modes
+    full = 0
+    while full + 32 <= len(p1) and len(set(hub[p1[full:full + 32]].tolist())) == 1 and hub[p1[full]] >= 0:
+        full += 32
+    np.testing.assert_array_equal(p1[:full], p2[:full])
+    # anchors of the hubbed tail are non-increasing in degree (each anchor one run)
+    h2, _ = planner.hubs(off, adj, np.where(hub >= 0, hub, 0), 128)
+    tail = [r for r in p2[full:] if sdeg[r] > 0 and hub[r] >= 0]
+    anchors = []
+    for r in tail:
+        a, b = hub[r], h2[r]
+        anchors.append(b if b >= 0 and (deg[b] > deg[a] or (deg[b] == deg[a] and b < a)) else a)
+    runs = [anchors[0]] + [y for x, y in zip(anchors, anchors[1:]) if y != x]
+    assert len(runs) == len(set(runs))
+    assert all(deg[x] >= deg[y] for x, y in zip(runs, runs[1:]))

@@ -12,7 +12,7 @@ cfg = ibfs_gen.CONFIGS[name]
 el = cfg.edges(threads=os.cpu_count())
 g = P.Graph.from_edgelist(el)
 src = cfg.sources(el)
-s = src[g.plan(src, 128)]
+s = src[g.plan(src, 128, hops=int(os.environ.get("PROBE_HOPS", 1)))]
 out = torch.empty((G * 128, g.nv), dtype=torch.int8, device="cuda")
 kw = {}
 for k, v in extra.items():

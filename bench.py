@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--alpha", type=float, default=4.0)
     ap.add_argument("--beta", type=float, default=24.0)
     ap.add_argument("--split-div", type=float, default=64.0)
+    ap.add_argument("--group-bits", type=int, default=0, help="instances per group (0 = the config's, 128)")
     ap.add_argument("--plan-hops", type=int, default=1, help="GroupBy hub radius (1 = the paper's steps, 2 = 2-hop anchors)")
     ap.add_argument("--max-depth", type=int, default=0, help="k-hop mode (the 3-hop index of §8.7): 0 = plain BFS")
     ap.add_argument("--no-e2e", action="store_true")
@@ -168,8 +169,8 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     cfg = ibfs_gen.CONFIGS[args.config]
-    W = cfg.group_bits
-    G = args.groups_per_rank or DEFAULT_GROUPS[args.config]
+    W = args.group_bits or cfg.group_bits
+    G = args.groups_per_rank or DEFAULT_GROUPS[args.config] * (cfg.group_bits // W)
 
     # ---- setup (untimed: timing starts with the data in GPU memory) ----------
     t0 = time.perf_counter()

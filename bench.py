@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--beta", type=float, default=24.0)
     ap.add_argument("--split-div", type=float, default=64.0)
     ap.add_argument("--group-bits", type=int, default=0, help="instances per group (0 = the config's, 128)")
-    ap.add_argument("--plan-hops", type=int, default=1, help="GroupBy hub radius (1 = the paper's steps, 2 = 2-hop anchors)")
+    ap.add_argument("--plan-hops", type=int, default=2, help="GroupBy hub radius (1 = the literal steps, 2 = 2-hop anchors, P:L577)")
     ap.add_argument("--max-depth", type=int, default=0, help="k-hop mode (the 3-hop index of §8.7): 0 = plain BFS")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -307,7 +307,7 @@ def main():
             "config": {"workload": cfg.name + (f", {args.max_depth}-hop" if args.max_depth else ""), "generator": f"R-MAT/Kronecker (A,B,C)={cfg.abc}, seed {cfg.graph_seed}",
                        "scale": cfg.scale, "edgefactor": cfg.ef, "group_bits": W,
                        "sources_per_rank_per_step": G * W, "groups_per_rank_per_step": G,
-                       "planner": "GroupBy" + (f" (hops={args.plan_hops})" if args.plan_hops != 1 else ""), "direction": args.direction,
+                       "planner": f"GroupBy (hops={args.plan_hops})", "direction": args.direction,
                        "groups_in_flight": args.groups_in_flight or "auto",
                        "max_depth": args.max_depth or None,
                        "l2": ("flush 256 MiB between steps" if flush is not None

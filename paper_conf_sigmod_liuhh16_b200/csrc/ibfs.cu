@@ -890,7 +890,7 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
     for (uint32_t r = 0; r < n; ++r)
       if (hsrc[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
     for (uint32_t r = 0; r < n; ++r) hsrc[r] = host_compact_id(g, hsrc[r]);  // planner works on compacted ids
-    std::vector<uint32_t> hub(n, 0xffffffffu), sdeg(n, 0), anchor;
+    std::vector<uint32_t> hub(n, 0xffffffffu), sdeg(n, 0), anchor, hubx;
     if (pp.mode == 0) {
       uint32_t *d_src = nullptr, *d_hub = nullptr, *d_sdeg = nullptr;
       CK(cudaMalloc(&d_src, (size_t)n * 4));
@@ -907,7 +907,26 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
         // hub of each source's hub (the same search from the hub vertex); anchor = the
         // larger of the two by (degree desc, id asc)
         std::vector<uint32_t> hv(n), hub2(n, 0xffffffffu);
-        for (uint32_t r = 0; r < n; ++r) hv[r] = hub[r] == 0xffffffffu ? NO_VERTEX : hub[r];
+        // a source without a hub reaches the core through its max-degree neighbour m(r)
+        // (any degree, the P:L661 rule): its hub becomes hub(m(r))
+        for (uint32_t r = 0; r < n; ++r) hv[r] = (hub[r] == 0xffffffffu && sdeg[r] > 0) ? hsrc[r] : NO_VERTEX;
+        e = cudaMemcpy(d_src, hv.data(), (size_t)n * 4, cudaMemcpyHostToDevice);
+        if (e == cudaSuccess) {
+          hub_kernel<<<blocks, 256>>>(g->d_off, g->d_adj, g->d_deg, d_src, n, pp.q, 1, d_hub, d_sdeg);
+          e = cudaGetLastError();
+        }
+        if (e == cudaSuccess) e = cudaMemcpy(hv.data(), d_hub, (size_t)n * 4, cudaMemcpyDeviceToHost);
+        for (uint32_t r = 0; r < n; ++r) if (hv[r] == 0xffffffffu) hv[r] = NO_VERTEX;  // m(r)
+        if (e == cudaSuccess) e = cudaMemcpy(d_src, hv.data(), (size_t)n * 4, cudaMemcpyHostToDevice);
+        if (e == cudaSuccess) {
+          hub_kernel<<<blocks, 256>>>(g->d_off, g->d_adj, g->d_deg, d_src, n, pp.q, uniform, d_hub, d_sdeg);
+          e = cudaGetLastError();
+        }
+        if (e == cudaSuccess) e = cudaMemcpy(hub2.data(), d_hub, (size_t)n * 4, cudaMemcpyDeviceToHost);
+        hubx = hub;  // step 3 buckets by the 1-hop hub; the ordering uses the extended one
+        for (uint32_t r = 0; r < n; ++r)
+          if (hub[r] == 0xffffffffu && sdeg[r] > 0) hubx[r] = hub2[r];  // hub(m(r)) (or none)
+        for (uint32_t r = 0; r < n; ++r) hv[r] = hubx[r] == 0xffffffffu ? NO_VERTEX : hubx[r];
         e = cudaMemcpy(d_src, hv.data(), (size_t)n * 4, cudaMemcpyHostToDevice);
         if (e == cudaSuccess) {
           hub_kernel<<<blocks, 256>>>(g->d_off, g->d_adj, g->d_deg, d_src, n, pp.q, uniform, d_hub, d_sdeg);
@@ -916,7 +935,7 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
         if (e == cudaSuccess) e = cudaMemcpy(hub2.data(), d_hub, (size_t)n * 4, cudaMemcpyDeviceToHost);
         anchor.assign(n, 0xffffffffu);
         for (uint32_t r = 0; r < n; ++r) {
-          uint32_t a = hub[r];
+          uint32_t a = hubx[r];
           const uint32_t b = hub2[r];
           if (a != 0xffffffffu && b != 0xffffffffu) {
             const uint64_t da = g->h_off[a + 1] - g->h_off[a], db = g->h_off[b + 1] - g->h_off[b];
@@ -931,8 +950,9 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
       CK(e);
     }
     auto deg_of = [&](uint32_t x) -> uint64_t { return g->h_off[x + 1] - g->h_off[x]; };
-    ibfs::plan::make_plan(pp, group_bits, n, hub, sdeg, deg_of, out_perm,
-                          pp.mode == 0 && pp.hops == 2 ? &anchor : nullptr);
+    const bool two = pp.mode == 0 && pp.hops == 2;
+    ibfs::plan::make_plan(pp, group_bits, n, hub, sdeg, deg_of, out_perm, two ? &anchor : nullptr,
+                          two ? &hubx : nullptr);
   });
 }
 

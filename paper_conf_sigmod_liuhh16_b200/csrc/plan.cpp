@@ -36,7 +36,7 @@ void seeded_shuffle(std::vector<uint32_t> &items, uint64_t seed) {
 void make_plan(const ibfs_plan_params &pp, uint32_t group_bits, uint32_t n,
                const std::vector<uint32_t> &hub, const std::vector<uint32_t> &sdeg,
                const std::function<uint64_t(uint32_t)> &deg_of, uint32_t *out_perm,
-               const std::vector<uint32_t> *anchor) {
+               const std::vector<uint32_t> *anchor, const std::vector<uint32_t> *hubx) {
   std::vector<uint32_t> perm;
   perm.reserve(n);
   if (pp.mode == 2) {
@@ -85,14 +85,15 @@ void make_plan(const ibfs_plan_params &pp, uint32_t group_bits, uint32_t n,
     for (uint32_t r = 0; r < n; ++r) {
       if (bucketed[r]) continue;
       if (sdeg[r] == 0) perm.push_back(r);
-      else if (anchor && hub[r] != NO_HUB) late.push_back(r);
+      else if (anchor && (*hubx)[r] != NO_HUB) late.push_back(r);
       else other.push_back(r);
     }
     if (anchor) {
       // hops = 2 ("as long as within the first several levels"): the bucket
-      // leftovers, and the sources Rule 1 never admitted that still have a hub, ordered
-      // by their 2-hop anchor (the larger of hub(r) and hub(hub(r)): the core vertex they
-      // reach within two levels), then by hub, then by position
+      // leftovers, and the remaining sources that have a hub (or reach one through their
+      // max-degree neighbour m(r): hubx = hub(m(r))), ordered by their 2-hop anchor (the
+      // larger of hubx(r) and hub(hubx(r)): the core vertex they reach within two or three
+      // levels), then by hubx, then by position
       std::vector<uint32_t> rest;
       for (uint32_t h : order) {
         Bucket &b = buckets[h];
@@ -104,7 +105,8 @@ void make_plan(const ibfs_plan_params &pp, uint32_t group_bits, uint32_t n,
       std::stable_sort(rest.begin(), rest.end(), [&](uint32_t x, uint32_t y) {
         const uint32_t ax = (*anchor)[x], ay = (*anchor)[y];
         if (ax != ay) return by_degree(ax, ay);
-        if (hub[x] != hub[y]) return by_degree(hub[x], hub[y]);
+        const uint32_t hx = (*hubx)[x], hy = (*hubx)[y];
+        if (hx != hy) return by_degree(hx, hy);
         return pos[x] < pos[y];
       });
       perm.insert(perm.end(), rest.begin(), rest.end());

@@ -39,11 +39,23 @@ namespace ibfs {
 constexpr int BLOCK = 256;
 constexpr int NWARP = BLOCK / 32;
 constexpr int QL = 1024;         // light-queue entries per work item
-constexpr int QH = 32;           // heavy TD-queue entries per work item
-constexpr int QBH = 256;         // heavy BU-queue entries per work item
-constexpr int LIGHT_DEG = 32;    // degree <= LIGHT_DEG: light
-constexpr int HUB_T = 8192;      // degree > HUB_T: hub (chunked rows)
-constexpr int CHUNK = 8192;      // hub-row edges per work item
+#ifndef IBFS_QH
+#define IBFS_QH 32
+#endif
+#ifndef IBFS_QBH
+#define IBFS_QBH 256
+#endif
+#ifndef IBFS_LIGHT_DEG
+#define IBFS_LIGHT_DEG 32
+#endif
+#ifndef IBFS_HUB_T
+#define IBFS_HUB_T 8192
+#endif
+constexpr int QH = IBFS_QH;             // heavy TD-queue entries per work item
+constexpr int QBH = IBFS_QBH;           // heavy BU-queue entries per work item
+constexpr int LIGHT_DEG = IBFS_LIGHT_DEG;  // degree <= LIGHT_DEG: light
+constexpr int HUB_T = IBFS_HUB_T;       // degree > HUB_T: hub (chunked rows)
+constexpr int CHUNK = IBFS_HUB_T;       // hub-row edges per work item
 constexpr int MAXL = 130;        // level index 1..129 (129 only detects depth > 127)
 constexpr int MAX_G = 128;       // groups per launch batch
 constexpr unsigned FULL = 0xffffffffu;

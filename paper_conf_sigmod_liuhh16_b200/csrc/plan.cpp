@@ -103,6 +103,9 @@ void make_plan(const ibfs_plan_params &pp, uint32_t group_bits, uint32_t n,
       std::vector<uint32_t> pos(n, 0);
       for (uint32_t i = 0; i < rest.size(); ++i) pos[rest[i]] = i;
       std::stable_sort(rest.begin(), rest.end(), [&](uint32_t x, uint32_t y) {
+        // sources with a 1-hop hub first; those reached through m(r) (a level later) after
+        const bool lx = hub[x] == NO_HUB, ly = hub[y] == NO_HUB;
+        if (lx != ly) return !lx;
         const uint32_t ax = (*anchor)[x], ay = (*anchor)[y];
         if (ax != ay) return by_degree(ax, ay);
         const uint32_t hx = (*hubx)[x], hy = (*hubx)[y];

@@ -913,6 +913,7 @@ struct CommitSmem {
 // then holds the mask M of sampled vertices new for instance 32p + i) and weights them
 // by degree through the degree bit planes D_b = ballot(bit b of deg): sum_b popc(M & D_b) << b.
 constexpr int SAMPLE_TILES = 4;
+constexpr int SPLIT_HEAVY = 1024;  // frontier vertices above this degree are counted exactly
 
 // Commit of level lc for one tile of group g: the CVT * BLOCK vertices from `base`.
 // visited |= S_lc, zero slot lc + 1, build both JFQs of level lc + 1 -- top-down: vertices
@@ -1040,8 +1041,26 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
 #pragma unroll
     for (int cls = 0; cls < 4; ++cls) wc[cls] += __popc(bal[k][cls]);
   }
+  if (!sparse) {  // block-uniform
+    // heavy vertices (degree > SPLIT_HEAVY) enter the per-instance frontier edge counts
+    // exactly on every tile, in sampled units (d / SAMPLE): a hub-dominated frontier is
+    // not left to the 1/SAMPLE lottery; the light ones below are sampled
+#pragma unroll
+    for (int k = 0; k < CVT; ++k) {
+      const bool hv = !wzero(n[k]) && dg[k] > (uint32_t)SPLIT_HEAVY;
+      uint32_t hb = __ballot_sync(FULL, hv);
+      while (hb) {
+        const int src = __ffs(hb) - 1;
+        hb &= hb - 1;
+        const float dd = (float)__shfl_sync(FULL, dg[k], src) * (1.0f / (float)SAMPLE);
+#pragma unroll
+        for (int p = 0; p < WordBits<T>::value / 32; ++p)
+          if ((__shfl_sync(FULL, wpiece(n[k], p), src) >> lane) & 1u) bc[p] += dd;
+      }
+    }
+  }
   if (sample && !sparse) {  // block-uniform
-    const uint32_t d0 = wzero(n[0]) ? 0u : dg[0];
+    const uint32_t d0 = (wzero(n[0]) || dg[0] > (uint32_t)SPLIT_HEAVY) ? 0u : dg[0];
     const uint32_t dmax = __reduce_or_sync(FULL, d0);
     if (dmax) {
       const int nb = 32 - __clz(dmax);

@@ -1687,8 +1687,13 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
   __syncthreads();
   const T *vis = a.visited + (size_t)g * a.gstride;
   unsigned long long acc[NP];
+  uint32_t cnt[NP][8];  // popcounts per (piece, degree bit plane < 8), weighted at the end
 #pragma unroll
-  for (int p = 0; p < NP; ++p) acc[p] = 0;
+  for (int p = 0; p < NP; ++p) {
+    acc[p] = 0;
+#pragma unroll
+    for (int b = 0; b < 8; ++b) cnt[p][b] = 0;
+  }
   const size_t nvr = ((size_t)a.nva + 31) & ~(size_t)31;  // warp-uniform trip count
   for (size_t v = (size_t)blockIdx.x * BLOCK + tid; v < nvr; v += (size_t)gridDim.x * BLOCK) {
     const bool in = v < a.nva;
@@ -1702,11 +1707,11 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
     // degrees < 256 through their 8 bit planes; the few larger ones (hubs) one by one
     const bool heavy = d >= 256u;
     const uint32_t dl = heavy ? 0u : d;
-    const int nb = 32 - __clz(__reduce_or_sync(FULL, dl));
-    for (int b = 0; b < nb; ++b) {
+#pragma unroll
+    for (int b = 0; b < 8; ++b) {
       const uint32_t db = __ballot_sync(FULL, (dl >> b) & 1u);
 #pragma unroll
-      for (int p = 0; p < NP; ++p) acc[p] += (unsigned long long)__popc(m[p] & db) << b;
+      for (int p = 0; p < NP; ++p) cnt[p][b] += __popc(m[p] & db);
     }
     uint32_t hv = __ballot_sync(FULL, heavy && !wzero(x));
     while (hv) {
@@ -1719,8 +1724,11 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
     }
   }
 #pragma unroll
-  for (int p = 0; p < NP; ++p)
+  for (int p = 0; p < NP; ++p) {
+#pragma unroll
+    for (int b = 0; b < 8; ++b) acc[p] += (unsigned long long)cnt[p][b] << b;
     if (acc[p]) atomicAdd(&s_m[p * 32 + lane], acc[p]);
+  }
   __syncthreads();
   for (int j = tid; j < rows; j += BLOCK)
     if (s_m[j]) atomicAdd(&m_out[(size_t)g * W + j], s_m[j]);

@@ -40,16 +40,16 @@ constexpr int BLOCK = 256;
 constexpr int NWARP = BLOCK / 32;
 constexpr int QL = 1024;         // light-queue entries per work item
 #ifndef IBFS_QH
-#define IBFS_QH 32
+#define IBFS_QH 64
 #endif
 #ifndef IBFS_QBH
-#define IBFS_QBH 256
+#define IBFS_QBH 2048
 #endif
 #ifndef IBFS_LIGHT_DEG
-#define IBFS_LIGHT_DEG 32
+#define IBFS_LIGHT_DEG 64
 #endif
 #ifndef IBFS_HUB_T
-#define IBFS_HUB_T 8192
+#define IBFS_HUB_T 16384
 #endif
 constexpr int QH = IBFS_QH;             // heavy TD-queue entries per work item
 constexpr int QBH = IBFS_QBH;           // heavy BU-queue entries per work item

@@ -17,3 +17,7 @@ B="python bench.py --config c5 --steps 1 --warmup 0 --no-e2e --no-cpu-baseline"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:level_kernel -s 1 -c 3 -o "$OUT/level_kernel_c5" $B > "$OUT/ncu_level.log" 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:depth_kernel -s 0 -c 1 -o "$OUT/depth_kernel_c5" $B > "$OUT/ncu_depth.log" 2>&1
 echo done > "$OUT/DONE"
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
+  -k regex:'level_kernel|depth_kernel|init_|ms_kernel|iso_fix' --csv --log-file "$OUT/launches_c5.csv" \
+  python bench.py --config c5 --steps 8 --warmup 0 --no-e2e --no-cpu-baseline > "$OUT/launches_c5.log" 2>&1
+echo done2 > "$OUT/DONE2"

@@ -978,6 +978,18 @@ constexpr int LEVELS_PER_CHECK = 4;  // levels per polled chunk; two chunks stay
 struct DevCache {
   std::vector<cudaEvent_t> timed, untimed;
   void *pinned = nullptr;
+  void *stage = nullptr;  // pinned host staging of per-batch statistics (grown on demand)
+  size_t stage_bytes = 0;
+  void *host_stage(size_t bytes) {
+    if (bytes > stage_bytes) {
+      if (stage) cudaFreeHost(stage);
+      stage = nullptr;
+      stage_bytes = 0;
+      CK(cudaMallocHost(&stage, bytes));
+      stage_bytes = bytes;
+    }
+    return stage;
+  }
 };
 struct ThreadCache {
   std::vector<std::pair<int, DevCache>> devs;
@@ -986,6 +998,7 @@ struct ThreadCache {
       for (auto e : d.second.timed) cudaEventDestroy(e);
       for (auto e : d.second.untimed) cudaEventDestroy(e);
       if (d.second.pinned) cudaFreeHost(d.second.pinned);
+      if (d.second.stage) cudaFreeHost(d.second.stage);
     }
   }
   DevCache &get(int dev) {
@@ -1066,7 +1079,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   uint32_t *work_ctr = sc.get<uint32_t>(MAXL);
   uint32_t *flags = sc.get<uint32_t>(4);  // batch_done, range_err, grid barrier (count, generation)
   unsigned long long *tstamp = sc.get<unsigned long long>((size_t)MAXL * 3);
-  std::vector<unsigned long long> h_ts((size_t)MAXL * 3);
+
   unsigned long long *d_m = sc.get<unsigned long long>((size_t)G * W);
   unsigned long long *d_dig = sc.get<unsigned long long>((size_t)G * W);
   int8_t *staging = out_dev ? nullptr : sc.get<int8_t>((size_t)G * rows_bytes_per_group);
@@ -1075,8 +1088,15 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   DevCache &dc = t_cache.get(g->device);
   if (!dc.pinned) CK(cudaMallocHost(&dc.pinned, 4096));
   volatile uint32_t *h_done = (volatile uint32_t *)dc.pinned;  // [0..255] done slots, [256] range
-  std::vector<LevelStat> h_lstat((size_t)G * MAXL);
-  std::vector<unsigned long long> h_m((size_t)G * W), h_dig((size_t)G * W);
+  // statistics staging in pinned host memory: level stats [G][MAXL], stamps [MAXL][3],
+  // m_s and digests [G*W] each (only the levels a batch ran are copied)
+  const size_t st_lstat = (size_t)G * MAXL * sizeof(LevelStat), st_ts = (size_t)MAXL * 3 * 8,
+               st_m = (size_t)G * W * 8;
+  unsigned char *hst = (unsigned char *)dc.host_stage(st_lstat + st_ts + 2 * st_m);
+  LevelStat *h_lstat = (LevelStat *)hst;
+  unsigned long long *h_ts = (unsigned long long *)(hst + st_lstat);
+  unsigned long long *h_mp = (unsigned long long *)(hst + st_lstat + st_ts);
+  unsigned long long *h_digp = h_mp + (size_t)G * W;
 
   BatchArgs<T> a{};
   a.off = g->d_off;
@@ -1250,11 +1270,13 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     CK(cudaGetLastError());
     CK(cudaEventRecord(f1, stream));
     kfin.push_back({f0, f1});
-    CK(cudaMemcpyAsync(h_lstat.data(), lstat, (size_t)Gb * MAXL * sizeof(LevelStat), cudaMemcpyDeviceToHost, stream));
-    CK(cudaMemcpyAsync(h_ts.data(), tstamp, (size_t)MAXL * 3 * 8, cudaMemcpyDeviceToHost, stream));
-    CK(cudaMemcpyAsync(h_m.data(), d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
+    const int lrows = std::min(level + 1, MAXL);  // levels 0..level-1 ran (and level is a no-op)
+    CK(cudaMemcpy2DAsync(h_lstat, MAXL * sizeof(LevelStat), lstat, MAXL * sizeof(LevelStat),
+                         (size_t)lrows * sizeof(LevelStat), Gb, cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(h_ts, tstamp, (size_t)lrows * 3 * 8, cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(h_mp, d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
     if (stats && stats->per_source_digest)
-      CK(cudaMemcpyAsync(h_dig.data(), d_dig, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
+      CK(cudaMemcpyAsync(h_digp, d_dig, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
     if (out_host) {
       cudaEvent_t c0 = timer.next(), c1 = timer.next();
       CK(cudaEventRecord(c0, stream));
@@ -1270,12 +1292,12 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     if (h_done[256]) range_error = true;
     // accumulate per-source outputs and statistics
     for (uint32_t r = 0; r < rows_in_batch; ++r) {
-      st.edges_traversed += h_m[r];
-      if (stats && stats->per_source_m) stats->per_source_m[(size_t)gb0 * W + r] = h_m[r];
-      if (stats && stats->per_source_digest) stats->per_source_digest[(size_t)gb0 * W + r] = h_dig[r];
+      st.edges_traversed += h_mp[r];
+      if (stats && stats->per_source_m) stats->per_source_m[(size_t)gb0 * W + r] = h_mp[r];
+      if (stats && stats->per_source_digest) stats->per_source_digest[(size_t)gb0 * W + r] = h_digp[r];
     }
     for (uint32_t gi = 0; gi < Gb; ++gi) {
-      for (int l = 1; l < MAXL; ++l) {
+      for (int l = 1; l < lrows; ++l) {
         const LevelStat &L = h_lstat[(size_t)gi * MAXL + l];
         if (L.dir == 0) continue;
         ibfs_level_stats &P = per_level[l - 1];
@@ -1298,7 +1320,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     }
     // phase times of each level kernel from its in-kernel globaltimer stamps: [first CTA
     // start, grid barrier, last CTA end]; the commit part belongs to level l-1
-    for (int l = 1; l < MAXL; ++l) {
+    for (int l = 1; l < lrows; ++l) {
       const unsigned long long t0 = h_ts[(size_t)l * 3], t1 = h_ts[(size_t)l * 3 + 1], t2 = h_ts[(size_t)l * 3 + 2];
       if (t0 == ~0ull || t1 < t0 || t2 < t1) continue;
       const double cms = (t1 - t0) * 1e-6, ems = (t2 - t1) * 1e-6;
@@ -1309,7 +1331,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         per_level[l - 2].commit_ms += cms;
       }
     }
-    for (int l = 1; l + 1 < MAXL; ++l) {  // idle between level l's last CTA and level l+1's first
+    for (int l = 1; l + 1 < lrows; ++l) {  // idle between level l's last CTA and level l+1's first
       const unsigned long long e = h_ts[(size_t)l * 3 + 2], b = h_ts[(size_t)(l + 1) * 3];
       if (e && b != ~0ull && b > e) st.level_gap_ms += (b - e) * 1e-6;
     }

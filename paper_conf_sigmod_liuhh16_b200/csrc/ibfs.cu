@@ -1072,6 +1072,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   const uint32_t nchunk32 = (nva + 31) / 32;
   uint8_t *dirty = sc.get<uint8_t>((size_t)G * std::max<uint32_t>(nchunk32, 1));
+  const uint32_t late_cap = nva / 32 + 1024;  // new vertices of sparse levels (per group)
+  unsigned long long *late = sc.get<unsigned long long>((size_t)G * late_cap);
+  uint32_t *late_n = sc.get<uint32_t>(G);
   const uint32_t chq_stride = std::max<uint32_t>(std::max(g->n_chunks, g->n_rchunks), 1);
   uint32_t *chq = sc.get<uint32_t>((size_t)G * 2 * chq_stride);
   GroupCtrl<T> *ctrl = sc.get<GroupCtrl<T>>(G);
@@ -1139,6 +1142,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.buq = buq;
   a.dirty = dirty;
   a.nchunk32 = nchunk32;
+  a.late = late;
+  a.late_n = late_n;
+  a.late_cap = late_cap;
   a.n_iso = nv - nva;
   a.pol.mode = o.direction;
   a.pol.bu_from = o.bu_from;
@@ -1173,6 +1179,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     a.out = out_dev ? out_depths + (size_t)gb0 * rows_bytes_per_group : staging;
     const uint32_t rows_in_batch = std::min<uint32_t>(Gb * W, n - gb0 * W);
     CK(cudaMemsetAsync(flags, 0, 4, stream));
+    CK(cudaMemsetAsync(late_n, 0, (size_t)G * 4, stream));
     CK(cudaMemsetAsync(d_m, 0, (size_t)G * W * 8, stream));  // m_s accumulates in ms_kernel
     cudaEvent_t w0 = timer.next(), w1 = timer.next();
     CK(cudaEventRecord(w0, stream));
@@ -1200,9 +1207,11 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
                                                                          std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DEPTH_MINB / Gb)));
       const int first = flushed < 0 ? 1 : 0;
       depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
-      launches++;
+      late_fix_kernel<T><<<dim3(std::min<uint32_t>((late_cap + 255) / 256, 64), Gb), 256, 0, stream>>>(a, flushed + 1, l1);
+      launches += 2;
       st.depth_launches++;
-      st.depth_bytes += (uint64_t)Gb * nva * (B * (uint64_t)(l1 - flushed)) + (uint64_t)rows_in_batch * nv;
+      // level-0 snapshots are never read (the sources come from the source list)
+      st.depth_bytes += (uint64_t)Gb * nva * (B * (uint64_t)(l1 - flushed - (first ? 1 : 0))) + (uint64_t)rows_in_batch * nv;
       if (first && batch_iso) {
         iso_fix_kernel<T><<<Gb, 128, 0, stream>>>(a);
         launches++;
@@ -1316,6 +1325,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         uint64_t cb = (uint64_t)nva * (3 * B + 4) + B * L.nf;
         st.expand_bytes += eb;
         st.commit_bytes += cb;
+        // a skipped level's snapshot is not read by the depth kernel; its new vertices
+        // (<= nf) are read back once from the late list by late_fix_kernel
+        if (L.skipped) st.depth_bytes -= (uint64_t)nva * B - (uint64_t)L.nf * (B + 8);
       }
     }
     // phase times of each level kernel from its in-kernel globaltimer stamps: [first CTA

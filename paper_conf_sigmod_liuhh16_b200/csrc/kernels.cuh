@@ -81,7 +81,8 @@ struct HubChunk {
 // Per group per level counters (device).  dir: 0 = level not run, 1 = TD, 2 = BU.
 struct LevelStat {
   unsigned long long jfq, fq, proc, insp, writes, newp, nf;
-  uint32_t dir, pad;
+  uint32_t dir;
+  uint32_t skipped;  // the depth kernel skips this level's snapshot (late list + fix-up)
 };
 
 template <typename T>
@@ -99,7 +100,11 @@ struct GroupCtrl {
   // per-instance direction split of a bottom-up level (include/ibfs.h IBFS_SPLIT_*):
   // td_bits = the active instances expanded top-down in the next level when dir == BU
   T td_bits;
-  uint32_t sparse;  // the last commit was sparse (no bottom-up queue: the next level is TD)  // the last commit was sparse (no bottom-up queue: the next level is TD)
+  uint32_t sparse;  // the last commit was sparse (no bottom-up queue: the next level is TD)
+  // levels whose snapshot the depth kernel does not read (bit l): level 0 (the sources,
+  // written by late_fix_kernel from the source list) and every sparse-committed level,
+  // whose few new vertices went to the late list instead
+  unsigned long long skip_lv[2];
   float bitw[WordBits<T>::value];  // sampled degree sum of the new frontier per instance (commit)
   float cumw[WordBits<T>::value];  // running sum of bitw over the levels so far (visited edges)
 };
@@ -139,6 +144,9 @@ struct BatchArgs {
   int gcap;      // groups allocated per slot
   uint32_t *tdq, *buq;  // [gcap][nva] queues
   uint8_t *dirty;       // [gcap][nchunk32] 32-vertex chunk of S_l written by a top-down RED.OR
+  unsigned long long *late;  // [gcap][late_cap] (level << 32 | v) new vertices of sparse commits
+  uint32_t *late_n;          // [gcap] appended entries (may exceed late_cap: then no more skips)
+  uint32_t late_cap;
   uint32_t nchunk32;    // ceil(nva / 32)
   GroupCtrl<T> *ctrl;
   LevelStat *lstat;     // [G][MAXL]
@@ -332,6 +340,8 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     c.last_level = done ? 0xffffffffu : 0u;  // done at init: no snapshot was ever written
     c.td_bits = wzero_value<T>();
     c.sparse = 0;
+    c.skip_lv[0] = 1ull;  // level 0: the sources (late_fix_kernel)
+    c.skip_lv[1] = 0ull;
     for (int j = 0; j < W; ++j) c.bitw[j] = c.cumw[j] = 0.f;
     a.ctrl[g] = c;
     if (rows > 0) {
@@ -1014,6 +1024,18 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
     }
     const bool nz = !wzero(n[k]);
     if (nz) st(vis + v, wor(vv[k], n[k]));
+    if (sparse) {  // block-uniform: the new vertices of a sparse level go to the late list
+      const uint32_t lb = __ballot_sync(FULL, nz);
+      if (lb) {
+        const int leader = __ffs(lb) - 1;
+        uint32_t base0 = 0;
+        if (lane == leader) base0 = atomicAdd(a.late_n + g, (uint32_t)__popc(lb));
+        base0 = __shfl_sync(FULL, base0, leader);
+        const uint32_t i = base0 + __popc(lb & lanemask_lt());
+        if (nz && i < a.late_cap)
+          a.late[(size_t)g * a.late_cap + i] = ((unsigned long long)lc << 32) | (unsigned long long)v;
+      }
+    }
     const T tp = (in && !sparse) ? wandn(active, wor(vv[k], n[k])) : wzero_value<T>();
     const bool un = !wzero(tp);
     const uint32_t d = dg[k], rd = rdg[k];
@@ -1203,6 +1225,10 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
     c->sparse = sparse ? 1u : 0u;
+    if (sparse && lc < 128 && *(volatile uint32_t *)(a.late_n + g) <= a.late_cap) {
+      c->skip_lv[lc >> 6] |= 1ull << (lc & 63);
+      ls->skipped = 1;
+    }
     c->last_level = (uint32_t)lc;
     for (int k = 0; k < NQ; ++k) c->qlen[(lc + 1) & 1][k] = 0;  // target of commit lc+1
     if (wzero(act) || (a.pol.max_depth != 0 && (uint32_t)lc >= a.pol.max_depth)) {
@@ -1483,6 +1509,8 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
   const GroupCtrl<T> *c = a.ctrl + g;
   const int last = min((int)c->last_level, min(l1, 127));
   const int nlev = last - l0 + 1;  // levels to read (may be <= 0)
+  const unsigned long long sk0 = c->skip_lv[0], sk1 = c->skip_lv[1];
+  auto skipped = [&](int l) { return ((l < 64 ? sk0 >> l : sk1 >> (l - 64)) & 1ull) != 0; };
   if (nlev <= 0 && !first) return;
   const int nbat = nlev > 0 ? (nlev + DLB - 1) / DLB : 1;  // >= 1 job per tile (its header)
   const size_t nvv = a.nv;
@@ -1536,10 +1564,13 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
         sts128(sb, k, off, c0, 0u);
         sts128(sb + 16, nzw.x, nzw.y, nzw.z, nzw.w);
       }
-      const uint32_t total = size * (uint32_t)nl;
+      uint32_t nread = 0;  // levels of this stage whose snapshot is read (the rest are skipped)
+      for (int l = lb; l <= le; ++l) nread += skipped(l) ? 0u : 1u;
+      const uint32_t total = size * nread;
       if (lane == 0) mbar_arrive_expect_tx(&s_full[st], total); else mbar_arrive(&s_full[st]);
       if (lane == 0)
         for (int l = lb; l <= le && total; ++l) {
+          if (skipped(l)) continue;
           const unsigned char *src = reinterpret_cast<const unsigned char *>(snap(a, g, l) + c0) - off;
           bulk_g2s(sb + DHDR + (uint32_t)((l - lb) * L::SROW), src, size, &s_full[st]);
         }
@@ -1588,6 +1619,7 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
 #pragma unroll
             for (int u = 0; u < DLB; ++u) {
               if (lb + u > le) break;
+              if (skipped(lb + u)) continue;  // not loaded: late_fix_kernel writes those depths
               const uint32_t hb = lds_part<PB>(p + (uint32_t)(u * L::SROW)) & ~reached[r];
               if (!hb) continue;
               const uint32_t inc = (uint32_t)(lb + u + 1);
@@ -1744,6 +1776,61 @@ __global__ void iso_fix_kernel(BatchArgs<T> a) {
   for (int j = threadIdx.x; j < rows; j += blockDim.x)
     if (a.csrc[(size_t)g * W + j] == NO_VERTEX)
       a.out[((size_t)g * W + j) * a.nv + a.src[(size_t)g * W + j]] = 0;
+}
+
+// Depths of the levels the depth kernel skipped (GroupCtrl::skip_lv), in [l0, l1]:
+// level 0 from the source list, the sparse-committed levels from the late list -- each
+// entry (l, v) writes l into the byte of every instance whose bit is in S_l[v].  Runs
+// after depth_kernel of the same flush (its first pass wrote -1 there).
+__device__ __forceinline__ uint32_t caller_id(const uint32_t *tbase, const uint32_t *nzbits, uint32_t ntiles,
+                                              uint32_t v) {
+  uint32_t lo = 0, hi = ntiles;  // last 128-column tile with tbase <= v
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(tbase + mid) <= v) lo = mid; else hi = mid;
+  }
+  uint32_t r = v - __ldg(tbase + lo);
+  for (uint32_t w = 4 * lo;; ++w) {
+    const uint32_t m = __ldg(nzbits + w), c = __popc(m);
+    if (r < c) return 32 * w + __fns(m, 0, (int)r + 1);
+    r -= c;
+  }
+}
+
+template <typename T>
+__global__ void late_fix_kernel(BatchArgs<T> a, int l0, int l1) {
+  constexpr int W = WordBits<T>::value;
+  const int g = blockIdx.y;
+  const int rows = group_rows(a, g);
+  if (rows == 0) return;
+  const GroupCtrl<T> *c = a.ctrl + g;
+  if (c->last_level == 0xffffffffu) return;  // done at init: nothing was traversed
+  const int last = min((int)c->last_level, min(l1, 127));
+  const unsigned long long sk0 = c->skip_lv[0], sk1 = c->skip_lv[1];
+  auto skipped = [&](int l) { return ((l < 64 ? sk0 >> l : sk1 >> (l - 64)) & 1ull) != 0; };
+  const size_t nvv = a.nv;
+  if (l0 == 0 && skipped(0) && blockIdx.x == 0)
+    for (int j = threadIdx.x; j < rows; j += blockDim.x)
+      if (a.csrc[(size_t)g * W + j] != NO_VERTEX) a.out[((size_t)g * W + j) * nvv + a.src[(size_t)g * W + j]] = 0;
+  const uint32_t n = min(a.late_n[g], a.late_cap);
+  const uint32_t ntiles = (uint32_t)((nvv + 127) / 128);
+  for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
+    const unsigned long long ent = a.late[(size_t)g * a.late_cap + e];
+    const int l = (int)(ent >> 32);
+    const uint32_t v = (uint32_t)ent;
+    if (l < l0 || l > last || !skipped(l)) continue;
+    const T x = ldg(snap(a, g, l) + v);
+    const size_t col = caller_id(a.tbase, a.nzbits, ntiles, v);
+#pragma unroll
+    for (int p = 0; p < W / 32; ++p) {
+      uint32_t m = wpiece(x, p);
+      while (m) {
+        const int j = 32 * p + __ffs(m) - 1;
+        m &= m - 1;
+        if (j < rows) a.out[((size_t)g * W + j) * nvv + col] = (int8_t)l;
+      }
+    }
+  }
 }
 
 __device__ __forceinline__ unsigned long long splitmix64(unsigned long long z) {

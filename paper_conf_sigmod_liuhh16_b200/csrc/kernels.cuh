@@ -39,6 +39,9 @@ namespace ibfs {
 constexpr int BLOCK = 256;
 constexpr int NWARP = BLOCK / 32;
 constexpr int QL = 1024;         // light-queue entries per work item
+#ifndef IBFS_DEPTH_SKIP
+#define IBFS_DEPTH_SKIP 1  // skip the level-0 and sparse-committed snapshots (A/B knob)
+#endif
 #ifndef IBFS_QH
 #define IBFS_QH 64
 #endif
@@ -340,7 +343,7 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     c.last_level = done ? 0xffffffffu : 0u;  // done at init: no snapshot was ever written
     c.td_bits = wzero_value<T>();
     c.sparse = 0;
-    c.skip_lv[0] = 1ull;  // level 0: the sources (late_fix_kernel)
+    c.skip_lv[0] = IBFS_DEPTH_SKIP ? 1ull : 0ull;  // level 0: the sources (late_fix_kernel)
     c.skip_lv[1] = 0ull;
     for (int j = 0; j < W; ++j) c.bitw[j] = c.cumw[j] = 0.f;
     a.ctrl[g] = c;
@@ -1225,7 +1228,7 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
     c->sparse = sparse ? 1u : 0u;
-    if (sparse && lc < 128 && *(volatile uint32_t *)(a.late_n + g) <= a.late_cap) {
+    if (IBFS_DEPTH_SKIP && sparse && lc < 128 && *(volatile uint32_t *)(a.late_n + g) <= a.late_cap) {
       c->skip_lv[lc >> 6] |= 1ull << (lc & 63);
       ls->skipped = 1;
     }
@@ -1384,7 +1387,7 @@ constexpr int DSLOTS = 64;            // dense slots per round (DTHREADS / 4 par
 #endif
 constexpr int DLB = IBFS_DEPTH_DLB;   // levels per pipeline stage
 constexpr int DNS = 3;                // pipeline stages
-constexpr int DHDR = 32 + DV;         // stage header: k, run offset, c0, pad, nzbits[4]; slot -> column table
+constexpr int DHDR = 32 + DV;         // stage header: k, run offset, c0, read mask, nzbits[4]; slot -> column table
 
 __device__ __forceinline__ uint32_t spread4(uint32_t nib) {
   // 4-bit nibble -> 0x01 in each byte whose bit is set
@@ -1560,17 +1563,17 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
           asm volatile("st.shared.u8 [%0], %1;" ::"r"(sb + 32 + pos), "h"((unsigned short)(4 * lane + cc)));
           ++pos;
         }
+      uint32_t rmask = 0;  // bit u: level lb + u is in range and its snapshot is loaded
+      for (int l = lb; l <= le; ++l) rmask |= skipped(l) ? 0u : 1u << (l - lb);
       if (lane == 0) {
-        sts128(sb, k, off, c0, 0u);
+        sts128(sb, k, off, c0, rmask);
         sts128(sb + 16, nzw.x, nzw.y, nzw.z, nzw.w);
       }
-      uint32_t nread = 0;  // levels of this stage whose snapshot is read (the rest are skipped)
-      for (int l = lb; l <= le; ++l) nread += skipped(l) ? 0u : 1u;
-      const uint32_t total = size * nread;
+      const uint32_t total = size * (uint32_t)__popc(rmask);
       if (lane == 0) mbar_arrive_expect_tx(&s_full[st], total); else mbar_arrive(&s_full[st]);
       if (lane == 0)
         for (int l = lb; l <= le && total; ++l) {
-          if (skipped(l)) continue;
+          if (!((rmask >> (l - lb)) & 1u)) continue;
           const unsigned char *src = reinterpret_cast<const unsigned char *>(snap(a, g, l) + c0) - off;
           bulk_g2s(sb + DHDR + (uint32_t)((l - lb) * L::SROW), src, size, &s_full[st]);
         }
@@ -1600,7 +1603,7 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
         const int st = (int)(job % DNS);
         mbar_wait(&s_full[st], (uint32_t)((job / DNS) & 1));
         const uint32_t sb = stage_base + (uint32_t)(st * L::STAGE);
-        const uint32_t off = lds32(sb + 4);
+        const uint32_t off = lds32(sb + 4), rm = lds32(sb + 12);  // rm: header's read mask
         if (b == 0) {
           k = lds32(sb);
           mynz = (lds32(sb + 16 + 4 * (col >> 5)) >> (col & 31)) & 1u;
@@ -1610,7 +1613,7 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
             if (i < k) dcol[r] = lds8(sb + 32 + i);
           }
         }
-        const int lb = l0 + b * DLB, le = min(last, lb + DLB - 1);
+        const int lb = l0 + b * DLB;
 #pragma unroll
         for (int r = 0; r < 2; ++r) {
           const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
@@ -1618,8 +1621,8 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
             const uint32_t p = sb + DHDR + off + i * (uint32_t)sizeof(T) + (uint32_t)(part * PB / 8);
 #pragma unroll
             for (int u = 0; u < DLB; ++u) {
-              if (lb + u > le) break;
-              if (skipped(lb + u)) continue;  // not loaded: late_fix_kernel writes those depths
+              // out of range, or not loaded (late_fix_kernel writes those depths)
+              if (!((rm >> u) & 1u)) continue;
               const uint32_t hb = lds_part<PB>(p + (uint32_t)(u * L::SROW)) & ~reached[r];
               if (!hb) continue;
               const uint32_t inc = (uint32_t)(lb + u + 1);

@@ -1375,15 +1375,6 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
 //     streaming stores -- the rows are written once and not re-read here).
 // first != 0 writes every byte; otherwise (a ring-slot flush before reuse) only the bytes
 // found in [l0, l1] change.  m_s and the isolated sources' own zero are separate passes.
-#ifndef IBFS_DEPTH_XOR
-#define IBFS_DEPTH_XOR 0
-#endif
-// IBFS_DEPTH_XOR: a depth byte starts at 0xff (-1) and its level l arrives as an XOR with
-// 0xff ^ l (each byte receives at most one value, so XOR sets it to l and no byte carries):
-// the store needs no per-byte l + 1 -> l subtraction.  Else it starts at 0 and accumulates
-// l + 1 (bytes never carry), turned into l (0 -> -1) by __vsub4 before the store.
-constexpr bool DXOR = IBFS_DEPTH_XOR != 0;
-constexpr uint32_t DACC0 = DXOR ? 0xFFFFFFFFu : 0u;  // an unreached depth byte in the accumulator
 constexpr int DV = 128;               // columns per tile
 constexpr int DCW = 8;                // consumer warps
 constexpr int DTHREADS = DCW * 32;    // consumer threads
@@ -1605,7 +1596,7 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
 #pragma unroll
       for (int r = 0; r < 2; ++r)
 #pragma unroll
-        for (int q = 0; q < PQ; ++q) acc[r][q] = DACC0;
+        for (int q = 0; q < PQ; ++q) acc[r][q] = 0;
       uint32_t reached[2] = {0u, 0u};
       uint32_t k = 0, mynz = 0, dcol[2] = {0u, 0u};
       for (int b = 0; b < nbat; ++b, ++job) {
@@ -1634,17 +1625,14 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
               if (!((rm >> u) & 1u)) continue;
               const uint32_t hb = lds_part<PB>(p + (uint32_t)(u * L::SROW)) & ~reached[r];
               if (!hb) continue;
-              const uint32_t inc = DXOR ? (uint32_t)(lb + u) ^ 0xFFu : (uint32_t)(lb + u + 1);
+              const uint32_t inc = (uint32_t)(lb + u + 1);
               if (reached[r] == 0u && hb == (PB == 32 ? 0xffffffffu : ((1u << PB) - 1u))) {
                 // the whole part at one level (common): no bit spreading
 #pragma unroll
-                for (int q = 0; q < PQ; ++q) acc[r][q] = (uint32_t)(lb + u + (DXOR ? 0 : 1)) * 0x01010101u;
+                for (int q = 0; q < PQ; ++q) acc[r][q] = inc * 0x01010101u;
               } else {
 #pragma unroll
-                for (int q = 0; q < PQ; ++q) {
-                  const uint32_t y = spread4((hb >> (4 * q)) & 0xFu) * inc;
-                  acc[r][q] = DXOR ? acc[r][q] ^ y : acc[r][q] + y;
-                }
+                for (int q = 0; q < PQ; ++q) acc[r][q] += spread4((hb >> (4 * q)) & 0xFu) * inc;
               }
               reached[r] |= hb;
             }
@@ -1682,27 +1670,22 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
         }
       } else {
 #pragma unroll
-        for (int q = 0; q < HW; ++q) x[q] = DACC0;
+        for (int q = 0; q < HW; ++q) x[q] = 0;
       }
       const size_t cbase = v0 + (size_t)(col & ~3);  // first column of this lane's quad
       const int row0 = half * (W / 2) + rowperm;
       int8_t *dst = a.out + ((size_t)g * W + row0) * nvv + cbase;  // row row0 + 4q at dst + 4q nv
       const bool fast = word_ok && v0 + DV <= nvv && first && rows == W;  // block-uniform
-      // 4 x 4 byte transpose among the lanes of a column quad: row row0 + 4q, 4 columns
-      auto quad_word = [&](int q) {
-        uint32_t w = DXOR ? x[q] : __vsub4(x[q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
+#pragma unroll
+      for (int q = 0; q < HW; ++q, dst += 4 * nvv) {
+        uint32_t w = __vsub4(x[q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
         uint32_t y = __shfl_xor_sync(FULL, w, 1);
         w = __byte_perm(w, y, sel1);
         y = __shfl_xor_sync(FULL, w, 2);
-        return __byte_perm(w, y, sel2);
-      };
-      if (fast) {  // block-uniform: the loop without per-word branches
-#pragma unroll
-        for (int q = 0; q < HW; ++q, dst += 4 * nvv) __stcs(reinterpret_cast<unsigned int *>(dst), quad_word(q));
-      } else {
-#pragma unroll
-        for (int q = 0; q < HW; ++q, dst += 4 * nvv) {
-          const uint32_t w = quad_word(q);
+        w = __byte_perm(w, y, sel2);
+        if (fast) {
+          __stcs(reinterpret_cast<unsigned int *>(dst), w);
+        } else {
           if (row0 + 4 * q >= rows) continue;
           const uint32_t ff = __vcmpeq4(w, 0xffffffffu);
           if (word_ok && v0 + DV <= nvv && ff == 0) {

@@ -122,7 +122,9 @@ void ibfs_plan_params_default(ibfs_plan_params *p);
  * into `sources` (host or device).  Group k = sources[out_perm[k*group_bits ..
  * k*group_bits + group_bits - 1]]; only the last group may be short.
  * *out_n_groups = ceil(n / group_bits).  group_bits in {32, 64, 128}.  params NULL =
- * defaults.  Runs a device kernel for the per-source hub search, the rest on the host. */
+ * defaults.  Runs a device kernel for the per-source hub search, the rest on the host.
+ * Device-resident `sources` are read after a device-wide synchronize (every stream's
+ * pending work, including the writer's, completes first). */
 int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
                      uint32_t group_bits, const ibfs_plan_params *params, uint32_t *out_perm,
                      uint32_t *out_n_groups);
@@ -161,7 +163,10 @@ typedef struct {
   float alpha;                /* TD->BU when m_f * alpha > m_u (default 4.0) */
   float beta;                 /* BU->TD when n_f * beta < nv_active (default 24.0) */
   uint32_t groups_in_flight;  /* groups per launch batch; 0 = auto from nv and memory */
-  void *cuda_stream;          /* cudaStream_t to launch on; NULL = legacy default stream */
+  void *cuda_stream;          /* cudaStream_t to launch on; NULL = legacy default stream.
+                                 Device-resident sources are read on this stream, so work
+                                 queued on it before the call (e.g. the kernel that wrote
+                                 them) completes first. */
   uint32_t timing;            /* 1: CUDA events around every level kernel -> stats */
   /* Per-instance direction inside a bottom-up level (never changes results).  The paper
      runs one direction per group; a BU level stops early at a vertex only
@@ -185,7 +190,12 @@ typedef struct {
      kept as the "Joint" rung of the ablation ladder (Fig. 15).  Same results
      (max_depth included); split and groups_in_flight are bitwise-engine options. */
   uint32_t engine;
-  uint32_t reserved[2];
+  /* Test hook: capacity of each group's late list -- the new vertices of sparse-committed
+     levels, whose depths are written by a fix-up pass instead of the depth kernel reading
+     their snapshot.  0 = default (non-isolated vertices / 32 + 1024).  A
+     level whose entries do not fit is read from its snapshot instead; results never change. */
+  uint32_t late_cap;
+  uint32_t reserved;
 } ibfs_run_opts;
 
 enum { IBFS_ENGINE_BITWISE = 0, IBFS_ENGINE_JOINT = 1 };
@@ -228,6 +238,23 @@ typedef struct {
   uint64_t expand_bytes, commit_bytes, init_bytes, depth_bytes;
   double level_gap_ms;  /* device idle between consecutive level kernels of a batch (in-kernel
                            globaltimer stamps): launch latency plus any host polling stall */
+  /* Byte models (SURVEY.md §8(d) "Algorithmic bytes"):
+     expand_bytes  per queued frontier 8 (row start) + B (its word); per inspection 4 + B
+                   (adjacency entry + the neighbour's word); per S_l write B;
+     commit_bytes  the §8(d) dense-scan model: 3B per vertex and level (S_l and visited
+                   read, the next slot cleared) + B per vertex with new bits;
+     commit_bytes_moved  what the commits actually stream: a sparse commit
+                   reads the chunk map, the marked chunks (bounded by the level's writes)
+                   and clears the next slot;
+     depth_bytes   depth_kernel only: int8 rows written (depth_rows_bytes) + B per vertex,
+                   group and loaded snapshot level (levels 1..last_level of each group,
+                   skipped levels excluded) + the late-list fix-ups;
+     ms_bytes      the m_s pass: (B + 4) per vertex and group (final words + degrees). */
+  uint64_t commit_bytes_moved, depth_rows_bytes, ms_bytes;
+  double ms_ms;                  /* m_s pass + late-list / isolated-source fix-ups (opts.timing) */
+  uint64_t ms_launches;
+  uint64_t level_launches_live;  /* level launches in which a group was still running (the
+                                    others are look-ahead launches that exit at once) */
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */
   uint64_t *per_source_digest;  /* [n] sum over reached v of splitmix64((v<<8)|(d+1)) */

@@ -15,7 +15,8 @@ Contents
   hand-built example: the depths do not depend on it).
 * ``stats``                  -- sharing degree (Eq. 1) and per-level frontier
   sizes, computed from depth rows.
-* ``certify``                -- the complete BFS-depth certificate.
+* ``certify``                -- the complete BFS-depth certificate (SURVEY.md App. C, C4);
+  ``OracleGraph.certify`` is the same certificate as C loops for full-size rows.
 """
 from __future__ import annotations
 
@@ -61,6 +62,8 @@ def _load():
         lib.oracle_bfs.argtypes = [P, P, ctypes.c_uint64, P, P, P, P, P, ctypes.c_int]
         lib.oracle_bfs_k.restype = ctypes.c_int
         lib.oracle_bfs_k.argtypes = [P, P, ctypes.c_uint64, ctypes.c_int32, P, P, P, P, P, ctypes.c_int]
+        lib.oracle_certify.restype = ctypes.c_int
+        lib.oracle_certify.argtypes = [P, ctypes.c_uint32, P]
         _lib = lib
     return _lib
 
@@ -145,6 +148,24 @@ class OracleGraph:
         if res.status not in (0, ORACLE_E_RANGE):
             raise ValueError(f"oracle_bfs failed: {res.status}")
         return res
+
+
+    CERTIFY_REASONS = {1: "(o) value < -1", 2: "(i) d(s) != 0", 3: "(ii) reachability differs across an edge",
+                       4: "(ii) |d(u)-d(v)| > 1 across an edge", 5: "(iii) a vertex other than s has depth 0",
+                       6: "(iii) a reached vertex has no neighbour one level closer"}
+
+    def certify(self, s: int, row) -> str | None:
+        """The complete certificate (certify.py's conditions, C loops; undirected graphs):
+        None if `row` is the exact BFS depth row from s, else the violated condition."""
+        if self.directed:
+            raise ValueError("the certificate is for undirected graphs")
+        d = np.ascontiguousarray(np.asarray(row), dtype=np.int8)
+        if d.shape != (self.nv,):
+            raise ValueError("row must have nv entries")
+        rc = _load().oracle_certify(self._h, int(s), d.ctypes.data)
+        if rc < 0:
+            raise ValueError("bad source")
+        return None if rc == 0 else self.CERTIFY_REASONS[rc]
 
 
 def bfs(el, sources, want_depths=True, threads=None, max_depth=None) -> OracleResult:

@@ -248,3 +248,34 @@ int oracle_bfs(const oracle_graph *g, const uint32_t *sources, uint64_t n, int8_
                uint64_t *m_s, uint64_t *digest, int32_t *ecc, uint64_t *reached, int threads) {
   return oracle_bfs_k(g, sources, n, -1, out, m_s, digest, ecc, reached, threads);
 }
+
+/* The complete BFS-depth certificate (the same four conditions as
+ * oracle/certify.py, written as plain loops over the oracle's own adjacency so it checks
+ * rows at config-5 scale).  Undirected graphs only.  Returns 0 if d is the exact BFS depth
+ * row from s, else the number of the first violated condition:
+ *   1 (o)   some d(v) < -1
+ *   2 (i)   d(s) != 0
+ *   3 (ii)  reachability differs across an edge
+ *   4 (ii)  |d(u) - d(v)| > 1 across an edge
+ *   5 (iii) a vertex other than s has depth 0
+ *   6 (iii) a reached vertex v != s has no neighbour at d(v) - 1 */
+int oracle_certify(const oracle_graph *g, uint32_t s, const int8_t *d) {
+  const uint64_t nv = g->nv;
+  if (s >= nv) return ORACLE_E_INVALID;
+  for (uint64_t v = 0; v < nv; ++v)
+    if (d[v] < -1) return 1;
+  if (d[s] != 0) return 2;
+  for (uint64_t u = 0; u < nv; ++u) {
+    const int du = d[u];
+    int has_pred = 0;
+    for (uint64_t k = g->off[u]; k < g->off[u + 1]; ++k) {
+      const int dv = d[g->adj[k]];
+      if ((du == -1) != (dv == -1)) return 3;
+      if (du >= 0 && (du - dv > 1 || dv - du > 1)) return 4;
+      if (du >= 1 && dv == du - 1) has_pred = 1;
+    }
+    if (du == 0 && u != s) return 5;
+    if (du >= 1 && !has_pred) return 6;
+  }
+  return 0;
+}

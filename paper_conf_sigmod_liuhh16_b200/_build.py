@@ -9,7 +9,14 @@ CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(os.path.dirname(HERE), "include")
 SO = os.path.join(HERE, "libibfs.so")
 SOURCES = ["ibfs.cu", "plan.cpp"]
-HEADERS = ["kernels.cuh", "word.cuh", "plan.h"]
+import glob as _glob
+
+
+def _headers():
+    """Every header the sources include (csrc/*.cuh, csrc/*.h), so an edit to any of
+    them rebuilds the library."""
+    return sorted(os.path.basename(p) for p in _glob.glob(os.path.join(CSRC, "*.cuh")) +
+                  _glob.glob(os.path.join(CSRC, "*.h")))
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
@@ -22,7 +29,7 @@ def _stale() -> bool:
     if not os.path.exists(SO):
         return True
     t = os.path.getmtime(SO)
-    deps = [os.path.join(CSRC, f) for f in SOURCES + HEADERS] + [os.path.join(INCLUDE, "ibfs.h")]
+    deps = [os.path.join(CSRC, f) for f in SOURCES + _headers()] + [os.path.join(INCLUDE, "ibfs.h")]
     return any(os.path.getmtime(d) > t for d in deps)
 
 

@@ -38,7 +38,8 @@ class RunOpts(C.Structure):
                 ("schedule_len", C.c_uint32), ("alpha", C.c_float), ("beta", C.c_float),
                 ("groups_in_flight", C.c_uint32), ("cuda_stream", C.c_void_p), ("timing", C.c_uint32),
                 ("split", C.c_uint32), ("split_mod", C.c_uint32), ("split_div", C.c_float),
-                ("max_depth", C.c_uint32), ("engine", C.c_uint32), ("reserved", C.c_uint32 * 2)]
+                ("max_depth", C.c_uint32), ("engine", C.c_uint32), ("late_cap", C.c_uint32),
+                ("reserved", C.c_uint32)]
 
 
 class LevelStats(C.Structure):
@@ -61,6 +62,8 @@ class Stats(C.Structure):
                 ("level_launches", C.c_uint64), ("init_launches", C.c_uint64), ("depth_launches", C.c_uint64),
                 ("expand_bytes", C.c_uint64), ("commit_bytes", C.c_uint64), ("init_bytes", C.c_uint64),
                 ("depth_bytes", C.c_uint64), ("level_gap_ms", C.c_double),
+                ("commit_bytes_moved", C.c_uint64), ("depth_rows_bytes", C.c_uint64), ("ms_bytes", C.c_uint64),
+                ("ms_ms", C.c_double), ("ms_launches", C.c_uint64), ("level_launches_live", C.c_uint64),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),
                 ("level_cap", C.c_uint32), ("per_level", C.c_void_p)]
 

@@ -886,6 +886,9 @@ extern "C" int ibfs_plan_groups(const ibfs_graph *g, const uint32_t *sources, ui
     if (n == 0) return;
     std::vector<uint32_t> hsrc(n);
     DeviceScope ds(g->device);
+    // device-resident sources: the caller completes the work that wrote them first
+    // (include/ibfs.h); a full device sync orders this read after every stream
+    if (is_device_ptr(sources)) CK(cudaDeviceSynchronize());
     CK(cudaMemcpy(hsrc.data(), sources, (size_t)n * 4, cudaMemcpyDefault));
     for (uint32_t r = 0; r < n; ++r)
       if (hsrc[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
@@ -1072,7 +1075,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   const uint32_t nchunk32 = (nva + 31) / 32;
   uint8_t *dirty = sc.get<uint8_t>((size_t)G * std::max<uint32_t>(nchunk32, 1));
-  const uint32_t late_cap = nva / 32 + 1024;  // new vertices of sparse levels (per group)
+  const uint32_t late_cap = o.late_cap ? o.late_cap : nva / 32 + 1024;  // new vertices of sparse levels (per group)
   unsigned long long *late = sc.get<unsigned long long>((size_t)G * late_cap);
   uint32_t *late_n = sc.get<uint32_t>(G);
   const uint32_t chq_stride = std::max<uint32_t>(std::max(g->n_chunks, g->n_rchunks), 1);
@@ -1164,7 +1167,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
 
   const int level_grid = g->num_sms * g->level_blocks_per_sm[W == 32 ? 0 : (W == 64 ? 1 : 2)];
   EventTimer timer(dc, true), chk(dc, false);
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin, kms;
   ibfs_stats st{};
   uint64_t launches = 0;
   bool range_error = false;
@@ -1201,29 +1204,35 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     bool batch_iso = false;  // a source of this batch is isolated (its own zero is a fix-up)
     for (uint32_t r = 0; r < rows_in_batch; ++r) batch_iso |= csources[(size_t)gb0 * W + r] == NO_VERTEX;
     auto flush = [&](int l1, bool final_flush) {
-      cudaEvent_t d0 = nullptr, d1 = nullptr;
+      cudaEvent_t d0 = nullptr, d1 = nullptr, m0 = nullptr, m1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
                                                                          std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DEPTH_MINB / Gb)));
       const int first = flushed < 0 ? 1 : 0;
       depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
-      late_fix_kernel<T><<<dim3(std::min<uint32_t>((late_cap + 255) / 256, 64), Gb), 256, 0, stream>>>(a, flushed + 1, l1);
-      launches += 2;
+      launches++;
       st.depth_launches++;
-      // level-0 snapshots are never read (the sources come from the source list)
-      st.depth_bytes += (uint64_t)Gb * nva * (B * (uint64_t)(l1 - flushed - (first ? 1 : 0))) + (uint64_t)rows_in_batch * nv;
+      // rows: each (instance, vertex) byte once per batch (§8(d) "i·|V| bytes"); the
+      // snapshot reads are counted per group from the level records after the batch
+      if (first) st.depth_rows_bytes += (uint64_t)rows_in_batch * nv;
+      if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); m0 = timer.next(); m1 = timer.next(); CK(cudaEventRecord(m0, stream)); }
+      late_fix_kernel<T><<<dim3(std::min<uint32_t>((late_cap + 255) / 256, 64), Gb), 256, 0, stream>>>(a, flushed + 1, l1);
+      launches++;
+      st.ms_launches++;
       if (first && batch_iso) {
         iso_fix_kernel<T><<<Gb, 128, 0, stream>>>(a);
         launches++;
+        st.ms_launches++;
       }
       if (final_flush) {  // m_s from the final visited words (reading #11)
         const uint32_t mx = (uint32_t)std::max<uint64_t>(
             1, std::min<uint64_t>(((uint64_t)nva + BLOCK - 1) / BLOCK, std::max<uint64_t>(1, (uint64_t)g->num_sms * 4 / Gb)));
         ms_kernel<T><<<dim3(mx, Gb), BLOCK, 0, stream>>>(a, d_m);
         launches++;
-        st.depth_bytes += (uint64_t)Gb * nva * (B + 4);
+        st.ms_launches++;
+        st.ms_bytes += (uint64_t)Gb * nva * (B + 4);
       }
-      if (o.timing) { CK(cudaEventRecord(d1, stream)); kdep.push_back({d0, d1}); }
+      if (o.timing) { CK(cudaEventRecord(m1, stream)); kms.push_back({m0, m1}); }
       flushed = l1;
     };
     int level = 1;
@@ -1317,19 +1326,33 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
         P.inspected += L.insp;
         P.new_pairs += L.newp;
         st.edges_inspected += L.insp;
-        // DESIGN.md §5 byte model
-        // expand: per queued frontier its queue entry, row start, degree and word; per
-        // inspection the adjacency entry and the neighbour's word; per write one word.
-        // commit: S_l, visited and the zeroed slot streamed, visited written where new.
-        uint64_t eb = (16 + B) * L.proc + (4 + B) * L.insp + B * L.writes;
-        uint64_t cb = (uint64_t)nva * (3 * B + 4) + B * L.nf;
+        // DESIGN.md §5 byte model (SURVEY.md §8(d) "Algorithmic bytes")
+        // expand: per queued frontier its row start and word; per inspection the adjacency
+        // entry and the neighbour's word; per S_l write one word.
+        // commit (§8(d) dense scan): S_l and visited read, the next slot cleared; visited
+        // written where new.
+        uint64_t eb = (8 + B) * L.proc + (4 + B) * L.insp + B * L.writes;
+        uint64_t cb = (uint64_t)nva * (3 * B) + B * L.nf;
         st.expand_bytes += eb;
         st.commit_bytes += cb;
-        // a skipped level's snapshot is not read by the depth kernel; its new vertices
-        // (<= nf) are read back once from the late list by late_fix_kernel
-        if (L.skipped) st.depth_bytes -= (uint64_t)nva * B - (uint64_t)L.nf * (B + 8);
+        // what the commit streams: dense -- S_l, visited, the cleared slot, degrees (and
+        // in-degrees), the chunk map; sparse -- the chunk map, the marked chunks (at most
+        // one per write) and the cleared slot
+        const uint64_t degb = g->directed ? 8 : 4;
+        if (L.flags & 2u) {
+          const uint64_t chunks = std::min<uint64_t>(L.writes, nchunk32);
+          st.commit_bytes_moved += nchunk32 + chunks * 32 * (2 * B + degb) + (uint64_t)nva * B + B * L.nf;
+        } else {
+          st.commit_bytes_moved += (uint64_t)nva * (3 * B + degb) + nchunk32 + B * L.nf;
+        }
+        // depth kernel: a loaded level's snapshot is read once; a skipped level's new
+        // vertices (<= nf) are read back from the late list (entry + word) instead
+        if (L.flags & 1u) st.depth_bytes += (uint64_t)L.nf * (B + 8);
+        else st.depth_bytes += (uint64_t)nva * B;
       }
     }
+    for (int l = 1; l < level; ++l)  // launches of levels 1..level-1 were queued
+      if (h_ts[(size_t)l * 3] != ~0ull) st.level_launches_live++;
     // phase times of each level kernel from its in-kernel globaltimer stamps: [first CTA
     // start, grid barrier, last CTA end]; the commit part belongs to level l-1
     for (int l = 1; l < lrows; ++l) {
@@ -1355,9 +1378,11 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   for (auto &p : kinit) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.init_ms += ms; }
   for (auto &p : kfin) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.finalize_ms += ms; }
   for (auto &p : kdep) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.depth_ms += ms; }
+  for (auto &p : kms) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.ms_ms += ms; }
+  st.depth_bytes += st.depth_rows_bytes;
   st.n_groups = n_groups;
   st.n_launches = launches;
-  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes + st.depth_bytes;
+  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes + st.depth_bytes + st.ms_bytes;
   if (stats) {
     st.per_source_m = stats->per_source_m;
     st.per_source_digest = stats->per_source_digest;
@@ -1558,9 +1583,12 @@ extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_
       return;
     }
     DeviceScope ds(g->device);
-    // sources: validate on the host
+    // sources: validate on the host.  Device-resident sources are read on the caller's
+    // stream (ordered after the work that wrote them; torch streams are non-blocking
+    // with respect to the legacy default stream)
     std::vector<uint32_t> hs(n), hcs(n);
-    CK(cudaMemcpy(hs.data(), sources, (size_t)n * 4, cudaMemcpyDefault));
+    CK(cudaMemcpyAsync(hs.data(), sources, (size_t)n * 4, cudaMemcpyDefault, (cudaStream_t)o.cuda_stream));
+    CK(cudaStreamSynchronize((cudaStream_t)o.cuda_stream));
     for (uint32_t r = 0; r < n; ++r)
       if (hs[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
     for (uint32_t r = 0; r < n; ++r) hcs[r] = host_compact_id(g, hs[r]);

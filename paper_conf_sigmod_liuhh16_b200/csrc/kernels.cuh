@@ -85,7 +85,8 @@ struct HubChunk {
 struct LevelStat {
   unsigned long long jfq, fq, proc, insp, writes, newp, nf;
   uint32_t dir;
-  uint32_t skipped;  // the depth kernel skips this level's snapshot (late list + fix-up)
+  uint32_t flags;    // bit 0: the depth kernel skips this level's snapshot (late list +
+                     // fix-up); bit 1: the level's commit was sparse
 };
 
 template <typename T>
@@ -356,7 +357,10 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
         l1->jfq = (unsigned long long)a.nv - (s_distinct == 1 ? 1u : 0u);
         l1->fq = (unsigned long long)rows * ((unsigned long long)a.nv - 1ull);
       }
-      if (done) l1->dir = first_dir + 1;  // level 1 "runs" and finds nothing
+      if (done) {  // level 1 "runs" and finds nothing; no snapshot is read for it
+        l1->dir = first_dir + 1;
+        l1->flags = 1u;
+      }
     }
     if (done) atomicAdd(a.batch_done, 1u);
   }
@@ -1228,9 +1232,10 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->td_filter = (double)c->vpairs * 2.0 > (double)a.nva * (double)wpopc(act) ? 1u : 0u;
     c->arrive = 0;
     c->sparse = sparse ? 1u : 0u;
+    ls->flags = sparse ? 2u : 0u;
     if (IBFS_DEPTH_SKIP && sparse && lc < 128 && *(volatile uint32_t *)(a.late_n + g) <= a.late_cap) {
       c->skip_lv[lc >> 6] |= 1ull << (lc & 63);
-      ls->skipped = 1;
+      ls->flags |= 1u;
     }
     c->last_level = (uint32_t)lc;
     for (int k = 0; k < NQ; ++k) c->qlen[(lc + 1) & 1][k] = 0;  // target of commit lc+1

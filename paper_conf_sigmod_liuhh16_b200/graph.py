@@ -89,6 +89,12 @@ class RunStats:
     init_bytes: int
     depth_bytes: int
     level_gap_ms: float
+    commit_bytes_moved: int
+    depth_rows_bytes: int
+    ms_bytes: int
+    ms_ms: float
+    ms_launches: int
+    level_launches_live: int
     per_source_m: np.ndarray | None = None
     per_source_digest: np.ndarray | None = None
     per_level: list = field(default_factory=list)
@@ -208,7 +214,7 @@ class Graph:
             groups_in_flight: int = 0, stream=None, timing: bool = False, want_m: bool = True,
             want_digest: bool = False, level_cap: int = 130, split: str = "auto",
             split_mod: int = 2, split_div: float = 64.0, max_depth: int | None = None,
-            engine: str = "bitwise"):
+            engine: str = "bitwise", late_cap: int = 0):
         """n concurrent BFS instances; returns (depths, RunStats).
 
         engine: "bitwise" (the product path) or "joint" (the byte-JSA joint traversal of §4,
@@ -266,6 +272,7 @@ class Graph:
                 raise ValueError("max_depth must be >= 1 (None = unbounded)")
             opts.max_depth = int(max_depth)
         opts.engine = {"bitwise": 0, "joint": 1}[engine]
+        opts.late_cap = int(late_cap)
         st = _lib.Stats()
         m_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_m else None
         d_arr = np.zeros(max(n, 1), dtype=np.uint64) if want_digest else None
@@ -285,6 +292,18 @@ class Graph:
             for i in range(min(level_cap, st.max_levels))
         ]
         return out, rs
+
+    def run_plain(self, sources, group_bits: int = 128, out=None):
+        """ibfs_run: the plain entry point north_star names (no options, no statistics; the
+        legacy default stream; returns after the work completes).  out: int8 [n, nv] host
+        (numpy / torch CPU) or device (torch CUDA) buffer, or None."""
+        lib = _lib.load()
+        src = _u32(sources)
+        n = _len(src)
+        ps, ks = _ptr(src)
+        po, ko = _ptr(out)
+        check(lib.ibfs_run(self._h, ps if n else None, n, int(group_bits), po))
+        return out
 
 
 def use_torch_allocator(enable: bool = True) -> None:

@@ -519,3 +519,37 @@ def test_joint_engine_configs(name):
     np.testing.assert_array_equal(d, ref.depths)
     np.testing.assert_array_equal(st.per_source_m, ref.m_s)
     np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+
+
+# ------------------------------------------ late-list overflow (depth-kernel skipping)
+@pytest.mark.parametrize("late_cap", [1, 7, 300])
+def test_late_list_overflow_falls_back_to_snapshots(late_cap):
+    # sparse-committed levels put their new vertices on a per-group late list instead of
+    # having the depth kernel read their snapshot.  A tiny late_cap makes
+    # the list overflow: the overflowing level (and every later sparse one) is read from
+    # its snapshot instead.  Results never change.  A 100-vertex path beside a 20,000-vertex random component: path sources discover one
+    # or two vertices per level, far below the sparse-commit threshold (writes <= nva/128)
+    rng = np.random.default_rng(77)
+    npath, ncomp = 100, 20000
+    pairs = [(i, i + 1) for i in range(npath - 1)]
+    pairs += [(npath + int(a), npath + int(b)) for a, b in rng.integers(0, ncomp, size=(3 * ncomp, 2))]
+    el = ibfs_gen.from_pairs(npath + ncomp, pairs)
+    g = P.Graph.from_edgelist(el)
+    src = np.concatenate([np.arange(0, npath, 3), npath + np.arange(0, 40)]).astype(np.uint32)
+    ref = oracle.bfs(el, src)
+    for W in (32, 128):
+        d, st = gpu_depths(g, src, W, late_cap=late_cap, want_digest=True)
+        np.testing.assert_array_equal(d, ref.depths)
+        np.testing.assert_array_equal(st.per_source_digest, ref.digest)
+        # the overflow path ran: fewer skipped snapshots -> more snapshot bytes read
+        _, st0 = gpu_depths(g, src, W, want_digest=True)
+        if late_cap < 100:
+            assert st.depth_bytes > st0.depth_bytes
+    cfg = ibfs_gen.CONFIGS["c2"]
+    el = cfg.edges()
+    s = cfg.sources(el)
+    g = P.Graph.from_edgelist(el)
+    d, st = gpu_depths(g, s, 128, late_cap=late_cap, want_digest=True)
+    ref = _oracle_c2(el, s)
+    np.testing.assert_array_equal(d, ref.depths)
+    np.testing.assert_array_equal(st.per_source_digest, ref.digest)

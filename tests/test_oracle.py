@@ -173,6 +173,35 @@ def test_certificate_accepts_oracle_and_rejects_perturbations():
     assert rejected > 100
 
 
+def test_c_certificate_matches_python_certificate():
+    # OracleGraph.certify (C loops, used on config-5 rows) vs certify.py on the same rows:
+    # both accept the oracle's rows and reject the same perturbations
+    rng = np.random.default_rng(11)
+    for trial in range(40):
+        nv = int(rng.integers(2, 50))
+        m = int(rng.integers(0, 3 * nv + 1))
+        pairs = [(int(rng.integers(nv)), int(rng.integers(nv))) for _ in range(m)]
+        el = ibfs_gen.from_pairs(nv, pairs if pairs else np.zeros((0, 2)))
+        g = oracle.OracleGraph.from_edges(el)
+        off, adj = g.adjacency()
+        srcs = rng.integers(0, nv, size=4).astype(np.uint32)
+        r = g.bfs(srcs)
+        for j, s in enumerate(srcs):
+            assert g.certify(int(s), r.depths[j]) is None
+            for _ in range(10):
+                row = r.depths[j].copy()
+                v = int(rng.integers(nv))
+                row[v] = np.int8(int(rng.choice([-2, -1, 0, 1, 2, 3, 7])))
+                py = certify.certify_row(off, adj, int(s), row)
+                c = g.certify(int(s), row)
+                assert (py is None) == (c is None), (trial, py, c)
+    # a closed form it must accept: path 0-1-...-9 from 0
+    el = ibfs_gen.from_pairs(10, [(i, i + 1) for i in range(9)])
+    g = oracle.OracleGraph.from_edges(el)
+    assert g.certify(0, np.arange(10, dtype=np.int8)) is None
+    assert g.certify(0, np.r_[np.arange(9), 7].astype(np.int8)) is not None
+
+
 def test_apsp_symmetry_and_mass():
     el = ibfs_gen.rmat(9, 8, ibfs_gen.KRONECKER, seed=5)
     g = oracle.OracleGraph.from_edges(el)

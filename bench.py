@@ -211,12 +211,12 @@ def make_roofline(config, sts, step_ms):
     rc = random_ceiling()
     if rc and exp_ms > 0:
         rate = insp / (exp_ms * 1e-3)
-        ceil = rc.get("gather16_per_s")
+        ceil = rc.get("gather16_per_s_2GiB")  # random 16-byte gathers over 2 GiB (4 c5 groups' words)
         rl["phases"]["level.expand"].update({
             "inspections_per_s": round(rate / 1e9, 3), "unit_rate": "G/s",
             "random_gather16_ceiling_per_s": round(ceil / 1e9, 3) if ceil else None,
             "frac_of_random_ceiling": round(rate / ceil, 4) if ceil else None,
-            "ceiling_source": rc.get("source")})
+            "ceiling_source": rc.get("source", "profiles/randbench.json")})
     return rl
 
 

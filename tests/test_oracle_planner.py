@@ -104,3 +104,39 @@ def test_groupby_hops2_invariants_and_anchor_order():
     runs = [anchors[0]] + [y for x, y in zip(anchors, anchors[1:]) if y != x]
     assert len(runs) == len(set(runs))
     assert all(deg[x] >= deg[y] for x, y in zip(runs, runs[1:]))
+
+
+def test_groupby_hops2_worked_example_by_hand():
+    """hops = 2 worked by hand from P:L577 ("it is not required that the source vertex
+    directly connects to a high-outdegree vertex, as long as within the first several
+    levels"), q = 3, p = (4,), W = 2.
+
+    Core hub H = 0 (deg 5: A, B, 20, 21, 22).  Hubs A = 1 (H, 10, 11, 12), B = 2 (H, 13, 23,
+    24), C = 3 (14, 25, 26, 27), all deg 4.  m = 12 (A, 15) has deg 2 <= q.  16 isolated;
+    17 - 18 a separate edge.
+    sources (index: vertex): 0:10  1:13  2:11  3:15  4:16  5:17  6:14
+      1-hop hubs: 10, 11 -> A; 13 -> B; 14 -> C; 15, 17 none (their neighbours have deg <= q)
+      step 3 (p = 4): buckets A [0, 2], B [1], C [6] visited A, B, C (deg 4 each, id asc);
+        A holds W = 2 -> group [0, 2]; leftovers [1] (B), [6] (C)
+      degree-0 sources: [4]
+      hubless 15: max-degree neighbour m(15) = 12, hub(12) = A -> hub 1, reached a level
+        later; 17: m(17) = 18, hub(18) none -> stays in the random remainder
+      2-hop anchors (larger of hub and hub(hub) by degree): 13 -> B -> hub(B) = H: anchor H;
+        14 -> C, hub(C) none: anchor C; 15 -> A -> hub(A) = H: anchor H
+      order: 1-hop hubbed first by anchor degree desc [1 (H), 6 (C)], then the m(r) ones [3]
+    perm = [0, 2] + [4] + [1, 6, 3] + shuffle([5]) = [0, 2, 4, 1, 6, 3, 5]."""
+    pairs = [(0, 1), (0, 2), (0, 20), (0, 21), (0, 22),
+             (1, 10), (1, 11), (1, 12),
+             (2, 13), (2, 23), (2, 24),
+             (3, 14), (3, 25), (3, 26), (3, 27),
+             (12, 15), (17, 18)]
+    off, adj = _csr(28, pairs)
+    deg = np.diff(off.astype(np.int64))
+    assert deg[[0, 1, 2, 3, 12]].tolist() == [5, 4, 4, 4, 2]
+    sources = np.array([10, 13, 11, 15, 16, 17, 14], dtype=np.uint32)
+    perm = planner.groupby(off, adj, sources, group_bits=2, q=3, p_list=(4,), hops=2)
+    assert perm.tolist() == [0, 2, 4, 1, 6, 3, 5]
+    # hops = 1 (the literal steps): leftovers in bucket order, then degree-0, then the
+    # random remainder {3, 5} (seeded order)
+    p1 = planner.groupby(off, adj, sources, group_bits=2, q=3, p_list=(4,), hops=1)
+    assert p1.tolist()[:5] == [0, 2, 1, 6, 4] and sorted(p1.tolist()[5:]) == [3, 5]

@@ -462,18 +462,27 @@ def cpu_baseline(el, sources, sample, max_depth=None):
     import oracle
     cores = host_cores()
     k = sample or cores
-    s = np.asarray(sources[:k], dtype=np.uint32)
     og = oracle.OracleGraph.from_edges(el)  # adjacency build: setup, untimed
-    t0 = time.perf_counter()
-    r = og.bfs(s, want_depths=False, threads=cores, max_depth=max_depth)
-    dt = time.perf_counter() - t0
-    t1 = time.perf_counter()
-    r1 = og.bfs(s[:1], want_depths=False, threads=1, max_depth=max_depth)
-    dt1 = time.perf_counter() - t1
+    while True:  # grow a too-short sample (small graphs) toward ~10 s of CPU work
+        s = np.asarray(sources[:k], dtype=np.uint32)
+        t0 = time.perf_counter()
+        r = og.bfs(s, want_depths=False, threads=cores, max_depth=max_depth)
+        dt = time.perf_counter() - t0
+        if sample or dt >= 2.0 or k >= len(sources):
+            break
+        k = min(len(sources), k * max(2, int(10.0 / max(dt, 1e-3))))
+    k1 = 1
+    while True:
+        t1 = time.perf_counter()
+        r1 = og.bfs(s[:k1], want_depths=False, threads=1, max_depth=max_depth)
+        dt1 = time.perf_counter() - t1
+        if dt1 >= 2.0 or k1 >= len(s):
+            break
+        k1 = min(len(s), k1 * max(2, int(5.0 / max(dt1, 1e-3))))
     return {"value": round(float(r.m_s.sum()) / dt / 1e9, 4), "unit": "GTEPS", "cores": min(cores, len(s)),
             "kind": "oracle", "seconds": round(dt, 2), "cpu_model": cpu_model(),
             "one_thread": {"value": round(float(r1.m_s.sum()) / dt1 / 1e9, 4), "unit": "GTEPS",
-                           "seconds": round(dt1, 2), "sample": "the first source of the sample"},
+                           "seconds": round(dt1, 2), "sample": f"the first {k1} source(s) of the sample"},
             "sample": f"{len(s)} sources of step 0 (textbook BFS each, one thread per source)"}
 
 

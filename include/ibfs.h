@@ -213,8 +213,10 @@ typedef struct {
   uint32_t td_groups, bu_groups;  /* groups that ran this level top-down / bottom-up */
   uint64_t jfq_td, fq_td;         /* |JFQ| and sum_j |FQ_j| of the TD groups (Eq. 1) */
   uint64_t jfq_bu, fq_bu;         /* same for the BU groups (reading #23) */
-  uint64_t inspected;             /* neighbour status words read */
+  uint64_t inspected;             /* neighbour inspections (adjacency entries examined) */
   uint64_t new_pairs;             /* (instance, vertex) pairs discovered (depth == l) */
+  uint64_t gathered;              /* neighbour status words actually read: bottom-up
+                                     frontier-bitmap hits + top-down pre-checks */
   double expand_ms, commit_ms;    /* device time of this level's launches (opts.timing) */
 } ibfs_level_stats;
 
@@ -239,10 +241,13 @@ typedef struct {
   double level_gap_ms;  /* device idle between consecutive level kernels of a batch (in-kernel
                            globaltimer stamps): launch latency plus any host polling stall */
   /* Byte models (SURVEY.md §8(d) "Algorithmic bytes"):
-     expand_bytes  per queued frontier 8 (row start) + B (its word); per inspection 4 + B
-                   (adjacency entry + the neighbour's word); per S_l write B;
+     expand_bytes  per queued frontier 8 (row start) + B (its word); per inspection 4
+                   (adjacency entry); per gathered neighbour word B (a bottom-up neighbour
+                   is read only when the frontier bitmap holds it); per S_l write B; a
+                   bottom-up level reads the frontier bitmap (nva/8) once;
      commit_bytes  the §8(d) dense-scan model: 3B per vertex and level (S_l and visited
-                   read, the next slot cleared) + B per vertex with new bits;
+                   read, the next slot cleared) + B per vertex with new bits + the frontier
+                   bitmap written (nva/8);
      commit_bytes_moved  what the commits actually stream: a sparse commit
                    reads the chunk map, the marked chunks (bounded by the level's writes)
                    and clears the next slot;
@@ -255,6 +260,7 @@ typedef struct {
   uint64_t ms_launches;
   uint64_t level_launches_live;  /* level launches in which a group was still running (the
                                     others are look-ahead launches that exit at once) */
+  uint64_t words_gathered;       /* sum of ibfs_level_stats.gathered */
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */
   uint64_t *per_source_digest;  /* [n] sum over reached v of splitmix64((v<<8)|(d+1)) */

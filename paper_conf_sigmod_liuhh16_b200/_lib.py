@@ -45,7 +45,7 @@ class RunOpts(C.Structure):
 class LevelStats(C.Structure):
     _fields_ = [("td_groups", C.c_uint32), ("bu_groups", C.c_uint32), ("jfq_td", C.c_uint64),
                 ("fq_td", C.c_uint64), ("jfq_bu", C.c_uint64), ("fq_bu", C.c_uint64),
-                ("inspected", C.c_uint64), ("new_pairs", C.c_uint64),
+                ("inspected", C.c_uint64), ("new_pairs", C.c_uint64), ("gathered", C.c_uint64),
                 ("expand_ms", C.c_double), ("commit_ms", C.c_double)]
 
 
@@ -64,6 +64,7 @@ class Stats(C.Structure):
                 ("depth_bytes", C.c_uint64), ("level_gap_ms", C.c_double),
                 ("commit_bytes_moved", C.c_uint64), ("depth_rows_bytes", C.c_uint64), ("ms_bytes", C.c_uint64),
                 ("ms_ms", C.c_double), ("ms_launches", C.c_uint64), ("level_launches_live", C.c_uint64),
+                ("words_gathered", C.c_uint64),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),
                 ("level_cap", C.c_uint32), ("per_level", C.c_void_p)]
 

@@ -12,6 +12,7 @@
 //   then m_s (+ digest) finalize outside the timed window; D2H of rows if the caller's
 //   buffer is on the host.
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 #include <cub/device/device_segmented_sort.cuh>
@@ -20,6 +21,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <mutex>
 #include <new>
 #include <string>
@@ -455,6 +457,12 @@ void finish_graph(ibfs_graph *g) {
                           (int)depth_smem_bytes<unsigned long long>()));
   CK(cudaFuncSetAttribute(depth_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                           (int)depth_smem_bytes<u128>()));
+  CK(cudaFuncSetAttribute(depth_tma_kernel<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)depth_tma_smem_bytes<uint32_t>()));
+  CK(cudaFuncSetAttribute(depth_tma_kernel<unsigned long long>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)depth_tma_smem_bytes<unsigned long long>()));
+  CK(cudaFuncSetAttribute(depth_tma_kernel<u128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                          (int)depth_tma_smem_bytes<u128>()));
   int occ = 1;
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_kernel<uint32_t>, BLOCK, sizeof(TileQueue<uint32_t>)));
   g->level_blocks_per_sm[0] = std::max(1, occ);
@@ -976,6 +984,54 @@ namespace {
 
 constexpr int LEVELS_PER_CHECK = 4;  // levels per polled chunk; two chunks stay queued ahead
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link).
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    cudaGetLastError();
+  });
+  return fn;
+}
+
+// Depth rows through 2-D TMA tensor stores (depth_tma_kernel) unless IBFS_DEPTH_TMA=0
+// (A/B runs) or the rows break the tensor map rules (row pitch nv and base 16-byte aligned).
+// Bottom-up frontier-bitmap probes: IBFS_BU_PROBE = 0 never, 1 when the frontier is small
+// (default), 2 always (A/B runs; results never change).
+uint32_t bu_probe_mode() {
+  static const uint32_t m = [] {
+    const char *e = std::getenv("IBFS_BU_PROBE");
+    return (e && e[0] >= '0' && e[0] <= '2') ? (uint32_t)(e[0] - '0') : 1u;
+  }();
+  return m;
+}
+
+bool depth_tma_enabled() {
+  static const bool on = [] {
+    const char *e = std::getenv("IBFS_DEPTH_TMA");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
+// Tensor map of a batch's rows: int8 [rows][nv] at `out`, boxes of DV columns x W rows.
+bool make_rows_tensor_map(CUtensorMap *m, int8_t *out, uint32_t nv, uint32_t rows, uint32_t W) {
+  PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
+  if (!enc || (nv % 16) != 0 || ((uintptr_t)out % 16) != 0 || rows == 0) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)nv, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)nv};
+  cuuint32_t box[2] = {(cuuint32_t)DV, (cuuint32_t)W};
+  cuuint32_t estr[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, out, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 // Per-thread, per-device cache of CUDA events and a pinned host word buffer: creating
 // them per call (cudaEventCreate, cudaMallocHost) costs far more than a small level.
 struct DevCache {
@@ -1075,6 +1131,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   const uint32_t nchunk32 = (nva + 31) / 32;
   uint8_t *dirty = sc.get<uint8_t>((size_t)G * std::max<uint32_t>(nchunk32, 1));
+  uint32_t *fbits = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nchunk32, 1));
   const uint32_t late_cap = o.late_cap ? o.late_cap : nva / 32 + 1024;  // new vertices of sparse levels (per group)
   unsigned long long *late = sc.get<unsigned long long>((size_t)G * late_cap);
   uint32_t *late_n = sc.get<uint32_t>(G);
@@ -1098,11 +1155,23 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   // m_s and digests [G*W] each (only the levels a batch ran are copied)
   const size_t st_lstat = (size_t)G * MAXL * sizeof(LevelStat), st_ts = (size_t)MAXL * 3 * 8,
                st_m = (size_t)G * W * 8;
-  unsigned char *hst = (unsigned char *)dc.host_stage(st_lstat + st_ts + 2 * st_m);
-  LevelStat *h_lstat = (LevelStat *)hst;
-  unsigned long long *h_ts = (unsigned long long *)(hst + st_lstat);
-  unsigned long long *h_mp = (unsigned long long *)(hst + st_lstat + st_ts);
-  unsigned long long *h_digp = h_mp + (size_t)G * W;
+  // two slots: batch b's statistics are copied into slot b % 2 and read on the host while
+  // batch b + 1 runs (no device idle between the batches of a call)
+  const size_t st_slot = ((st_lstat + st_ts + 2 * st_m + 16) + 255) & ~(size_t)255;
+  unsigned char *hst = (unsigned char *)dc.host_stage(2 * st_slot);
+  struct Slot {
+    LevelStat *lstat;
+    unsigned long long *ts, *m, *dig;
+    uint32_t *range;
+  } slots[2];
+  for (int k = 0; k < 2; ++k) {
+    unsigned char *b = hst + k * st_slot;
+    slots[k].lstat = (LevelStat *)b;
+    slots[k].ts = (unsigned long long *)(b + st_lstat);
+    slots[k].m = (unsigned long long *)(b + st_lstat + st_ts);
+    slots[k].dig = slots[k].m + (size_t)G * W;
+    slots[k].range = (uint32_t *)(slots[k].dig + (size_t)G * W);
+  }
 
   BatchArgs<T> a{};
   a.off = g->d_off;
@@ -1144,6 +1213,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.tdq = tdq;
   a.buq = buq;
   a.dirty = dirty;
+  a.fbits = fbits;
   a.nchunk32 = nchunk32;
   a.late = late;
   a.late_n = late_n;
@@ -1159,6 +1229,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   a.pol.split_mod = std::max<uint32_t>(1, o.split_mod);
   a.pol.split_div = o.split_div;
   a.pol.max_depth = o.max_depth;
+  a.pol.bu_probe = bu_probe_mode();
   a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
   for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
   uint32_t first_dir = 0;
@@ -1167,14 +1238,99 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
 
   const int level_grid = g->num_sms * g->level_blocks_per_sm[W == 32 ? 0 : (W == 64 ? 1 : 2)];
   EventTimer timer(dc, true), chk(dc, false);
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin, kms;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin, kms, kcopy;
   ibfs_stats st{};
   uint64_t launches = 0;
   bool range_error = false;
   std::vector<ibfs_level_stats> per_level(MAXL);
 
-  for (uint32_t gb0 = 0; gb0 < n_groups; gb0 += G) {
+  struct Pending {
+    bool valid = false;
+    uint32_t gb0 = 0, Gb = 0, rows = 0;
+    int level = 0, slot = 0;
+    cudaEvent_t done = nullptr;
+  } pend;
+  // host side of a finished batch: per-source outputs, level records, byte models, times
+  auto harvest = [&](const Pending &pb) {
+    CK(cudaEventSynchronize(pb.done));
+    const Slot &sl = slots[pb.slot];
+    const uint32_t gb0 = pb.gb0, Gb = pb.Gb, rows_in_batch = pb.rows;
+    const int level = pb.level;
+    const int lrows = std::min(level + 1, MAXL);
+    const LevelStat *h_lstat = sl.lstat;
+    const unsigned long long *h_ts = sl.ts, *h_mp = sl.m, *h_digp = sl.dig;
+    if (*sl.range) range_error = true;
+    // accumulate per-source outputs and statistics
+    for (uint32_t r = 0; r < rows_in_batch; ++r) {
+      st.edges_traversed += h_mp[r];
+      if (stats && stats->per_source_m) stats->per_source_m[(size_t)gb0 * W + r] = h_mp[r];
+      if (stats && stats->per_source_digest) stats->per_source_digest[(size_t)gb0 * W + r] = h_digp[r];
+    }
+    for (uint32_t gi = 0; gi < Gb; ++gi) {
+      for (int l = 1; l < lrows; ++l) {
+        const LevelStat &L = h_lstat[(size_t)gi * MAXL + l];
+        if (L.dir == 0) continue;
+        ibfs_level_stats &P = per_level[l - 1];
+        const bool td = L.dir == 1;
+        st.max_levels = std::max<uint32_t>(st.max_levels, (uint32_t)l);
+        if (td) { P.td_groups++; P.jfq_td += L.jfq; P.fq_td += L.fq; st.levels_td++; st.sd_fq_td += L.fq; st.sd_jfq_td += L.jfq; }
+        else { P.bu_groups++; P.jfq_bu += L.jfq; P.fq_bu += L.fq; st.levels_bu++; st.sd_fq_bu += L.fq; st.sd_jfq_bu += L.jfq; }
+        P.inspected += L.insp;
+        P.new_pairs += L.newp;
+        P.gathered += L.gath;
+        st.words_gathered += L.gath;
+        st.edges_inspected += L.insp;
+        // DESIGN.md §5 byte model (SURVEY.md §8(d) "Algorithmic bytes")
+        // expand: per queued frontier its row start and word; per inspection the adjacency
+        // entry (4 B); the neighbour's word (B) only when it is gathered -- a bottom-up
+        // frontier-bitmap hit or a top-down pre-check; per S_l write one
+        // word; a bottom-up level reads the group's frontier bitmap (nva / 8 B) once.
+        // commit (§8(d) dense scan): S_l and visited read, the next slot cleared, visited
+        // written where new, the frontier bitmap written (nva / 8 B).
+        uint64_t eb = (8 + B) * L.proc + 4 * L.insp + B * L.gath + B * L.writes + (L.dir == 2 ? (uint64_t)nchunk32 * 4 : 0);
+        uint64_t cb = (uint64_t)nva * (3 * B) + B * L.nf + (uint64_t)nchunk32 * 4;
+        st.expand_bytes += eb;
+        st.commit_bytes += cb;
+        // what the commit streams: dense -- S_l, visited, the cleared slot, degrees (and
+        // in-degrees), the chunk map; sparse -- the chunk map, the marked chunks (at most
+        // one per write) and the cleared slot
+        const uint64_t degb = g->directed ? 8 : 4;
+        if (L.flags & 2u) {
+          const uint64_t chunks = std::min<uint64_t>(L.writes, nchunk32);
+          st.commit_bytes_moved += nchunk32 * 5ull + chunks * 32 * (2 * B + degb) + (uint64_t)nva * B + B * L.nf;
+        } else {
+          st.commit_bytes_moved += (uint64_t)nva * (3 * B + degb) + nchunk32 * 5ull + B * L.nf;
+        }
+        // depth kernel: a loaded level's snapshot is read once; a skipped level's new
+        // vertices (<= nf) are read back from the late list (entry + word) instead
+        if (L.flags & 1u) st.depth_bytes += (uint64_t)L.nf * (B + 8);
+        else st.depth_bytes += (uint64_t)nva * B;
+      }
+    }
+    for (int l = 1; l < level; ++l)  // launches of levels 1..level-1 were queued
+      if (h_ts[(size_t)l * 3] != ~0ull) st.level_launches_live++;
+    // phase times of each level kernel from its in-kernel globaltimer stamps: [first CTA
+    // start, grid barrier, last CTA end]; the commit part belongs to level l-1
+    for (int l = 1; l < lrows; ++l) {
+      const unsigned long long t0 = h_ts[(size_t)l * 3], t1 = h_ts[(size_t)l * 3 + 1], t2 = h_ts[(size_t)l * 3 + 2];
+      if (t0 == ~0ull || t1 < t0 || t2 < t1) continue;
+      const double cms = (t1 - t0) * 1e-6, ems = (t2 - t1) * 1e-6;
+      st.expand_ms += ems;
+      per_level[l - 1].expand_ms += ems;
+      if (l > 1) {
+        st.commit_ms += cms;
+        per_level[l - 2].commit_ms += cms;
+      }
+    }
+    for (int l = 1; l + 1 < lrows; ++l) {  // idle between level l's last CTA and level l+1's first
+      const unsigned long long e = h_ts[(size_t)l * 3 + 2], b = h_ts[(size_t)(l + 1) * 3];
+      if (e && b != ~0ull && b > e) st.level_gap_ms += (b - e) * 1e-6;
+    }
+  };
+  int batch_no = 0;
+  for (uint32_t gb0 = 0; gb0 < n_groups; gb0 += G, ++batch_no) {
     const uint32_t Gb = std::min(G, n_groups - gb0);
+    const Slot &sl = slots[batch_no & 1];
     a.G = (int)Gb;
     a.group0 = gb0;
     a.src = d_src + (size_t)gb0 * W;
@@ -1209,7 +1365,14 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
                                                                          std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DEPTH_MINB / Gb)));
       const int first = flushed < 0 ? 1 : 0;
-      depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
+      CUtensorMap tmap;
+      if (first && depth_tma_enabled() && make_rows_tensor_map(&tmap, a.out, nv, rows_in_batch, W)) {
+        const uint32_t bt = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
+                                                                           std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DTMA_MINB / Gb)));
+        depth_tma_kernel<T><<<dim3(bt, Gb), DTHREADS + 32, depth_tma_smem_bytes<T>(), stream>>>(tmap, a, flushed + 1, l1);
+      } else {
+        depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
+      }
       launches++;
       st.depth_launches++;
       // rows: each (instance, vertex) byte once per batch (§8(d) "i·|V| bytes"); the
@@ -1275,7 +1438,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     CK(cudaEventRecord(w1, stream));
     win.push_back({w0, w1});
     // range check (a level-128 discovery means a depth > 127)
-    CK(cudaMemcpyAsync((void *)(h_done + 256), flags + 1, 4, cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(sl.range, flags + 1, 4, cudaMemcpyDeviceToHost, stream));
     // finalize: m_s and digests (outside the traversal window)
     cudaEvent_t f0 = timer.next(), f1 = timer.next();
     CK(cudaEventRecord(f0, stream));
@@ -1289,88 +1452,35 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     CK(cudaEventRecord(f1, stream));
     kfin.push_back({f0, f1});
     const int lrows = std::min(level + 1, MAXL);  // levels 0..level-1 ran (and level is a no-op)
-    CK(cudaMemcpy2DAsync(h_lstat, MAXL * sizeof(LevelStat), lstat, MAXL * sizeof(LevelStat),
+    CK(cudaMemcpy2DAsync(sl.lstat, MAXL * sizeof(LevelStat), lstat, MAXL * sizeof(LevelStat),
                          (size_t)lrows * sizeof(LevelStat), Gb, cudaMemcpyDeviceToHost, stream));
-    CK(cudaMemcpyAsync(h_ts, tstamp, (size_t)lrows * 3 * 8, cudaMemcpyDeviceToHost, stream));
-    CK(cudaMemcpyAsync(h_mp, d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(sl.ts, tstamp, (size_t)lrows * 3 * 8, cudaMemcpyDeviceToHost, stream));
+    CK(cudaMemcpyAsync(sl.m, d_m, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
     if (stats && stats->per_source_digest)
-      CK(cudaMemcpyAsync(h_digp, d_dig, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
-    if (out_host) {
+      CK(cudaMemcpyAsync(sl.dig, d_dig, (size_t)Gb * W * 8, cudaMemcpyDeviceToHost, stream));
+    if (out_host) {  // rows of a host buffer: D2H from the staging rows (stream-ordered
+                     // before the next batch's depth kernel rewrites them)
       cudaEvent_t c0 = timer.next(), c1 = timer.next();
       CK(cudaEventRecord(c0, stream));
       CK(cudaMemcpyAsync(out_depths + (size_t)gb0 * rows_bytes_per_group, staging,
                          (size_t)rows_in_batch * nv, cudaMemcpyDeviceToHost, stream));
       CK(cudaEventRecord(c1, stream));
-      CK(cudaStreamSynchronize(stream));
-      float ms = 0;
-      CK(cudaEventElapsedTime(&ms, c0, c1));
-      st.copyout_ms += ms;
+      kcopy.push_back({c0, c1});
     }
-    CK(cudaStreamSynchronize(stream));
-    if (h_done[256]) range_error = true;
-    // accumulate per-source outputs and statistics
-    for (uint32_t r = 0; r < rows_in_batch; ++r) {
-      st.edges_traversed += h_mp[r];
-      if (stats && stats->per_source_m) stats->per_source_m[(size_t)gb0 * W + r] = h_mp[r];
-      if (stats && stats->per_source_digest) stats->per_source_digest[(size_t)gb0 * W + r] = h_digp[r];
-    }
-    for (uint32_t gi = 0; gi < Gb; ++gi) {
-      for (int l = 1; l < lrows; ++l) {
-        const LevelStat &L = h_lstat[(size_t)gi * MAXL + l];
-        if (L.dir == 0) continue;
-        ibfs_level_stats &P = per_level[l - 1];
-        const bool td = L.dir == 1;
-        st.max_levels = std::max<uint32_t>(st.max_levels, (uint32_t)l);
-        if (td) { P.td_groups++; P.jfq_td += L.jfq; P.fq_td += L.fq; st.levels_td++; st.sd_fq_td += L.fq; st.sd_jfq_td += L.jfq; }
-        else { P.bu_groups++; P.jfq_bu += L.jfq; P.fq_bu += L.fq; st.levels_bu++; st.sd_fq_bu += L.fq; st.sd_jfq_bu += L.jfq; }
-        P.inspected += L.insp;
-        P.new_pairs += L.newp;
-        st.edges_inspected += L.insp;
-        // DESIGN.md §5 byte model (SURVEY.md §8(d) "Algorithmic bytes")
-        // expand: per queued frontier its row start and word; per inspection the adjacency
-        // entry and the neighbour's word; per S_l write one word.
-        // commit (§8(d) dense scan): S_l and visited read, the next slot cleared; visited
-        // written where new.
-        uint64_t eb = (8 + B) * L.proc + (4 + B) * L.insp + B * L.writes;
-        uint64_t cb = (uint64_t)nva * (3 * B) + B * L.nf;
-        st.expand_bytes += eb;
-        st.commit_bytes += cb;
-        // what the commit streams: dense -- S_l, visited, the cleared slot, degrees (and
-        // in-degrees), the chunk map; sparse -- the chunk map, the marked chunks (at most
-        // one per write) and the cleared slot
-        const uint64_t degb = g->directed ? 8 : 4;
-        if (L.flags & 2u) {
-          const uint64_t chunks = std::min<uint64_t>(L.writes, nchunk32);
-          st.commit_bytes_moved += nchunk32 + chunks * 32 * (2 * B + degb) + (uint64_t)nva * B + B * L.nf;
-        } else {
-          st.commit_bytes_moved += (uint64_t)nva * (3 * B + degb) + nchunk32 + B * L.nf;
-        }
-        // depth kernel: a loaded level's snapshot is read once; a skipped level's new
-        // vertices (<= nf) are read back from the late list (entry + word) instead
-        if (L.flags & 1u) st.depth_bytes += (uint64_t)L.nf * (B + 8);
-        else st.depth_bytes += (uint64_t)nva * B;
-      }
-    }
-    for (int l = 1; l < level; ++l)  // launches of levels 1..level-1 were queued
-      if (h_ts[(size_t)l * 3] != ~0ull) st.level_launches_live++;
-    // phase times of each level kernel from its in-kernel globaltimer stamps: [first CTA
-    // start, grid barrier, last CTA end]; the commit part belongs to level l-1
-    for (int l = 1; l < lrows; ++l) {
-      const unsigned long long t0 = h_ts[(size_t)l * 3], t1 = h_ts[(size_t)l * 3 + 1], t2 = h_ts[(size_t)l * 3 + 2];
-      if (t0 == ~0ull || t1 < t0 || t2 < t1) continue;
-      const double cms = (t1 - t0) * 1e-6, ems = (t2 - t1) * 1e-6;
-      st.expand_ms += ems;
-      per_level[l - 1].expand_ms += ems;
-      if (l > 1) {
-        st.commit_ms += cms;
-        per_level[l - 2].commit_ms += cms;
-      }
-    }
-    for (int l = 1; l + 1 < lrows; ++l) {  // idle between level l's last CTA and level l+1's first
-      const unsigned long long e = h_ts[(size_t)l * 3 + 2], b = h_ts[(size_t)(l + 1) * 3];
-      if (e && b != ~0ull && b > e) st.level_gap_ms += (b - e) * 1e-6;
-    }
+    Pending cur;
+    cur.valid = true;
+    cur.gb0 = gb0;
+    cur.Gb = Gb;
+    cur.rows = rows_in_batch;
+    cur.level = level;
+    cur.slot = batch_no & 1;
+    cur.done = timer.next();  // not from `chk`: its events are recycled every batch
+    CK(cudaEventRecord(cur.done, stream));
+    // the previous batch's statistics, while this one runs; its slot is reused next
+    if (pend.valid) harvest(pend);
+    pend = cur;
   }
+  if (pend.valid) harvest(pend);
   if (range_error) fail(IBFS_E_RANGE, "a depth exceeds 127 (int8 output)");
   // times
   for (auto &p : win) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.traverse_ms += ms; }
@@ -1379,6 +1489,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   for (auto &p : kfin) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.finalize_ms += ms; }
   for (auto &p : kdep) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.depth_ms += ms; }
   for (auto &p : kms) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.ms_ms += ms; }
+  for (auto &p : kcopy) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.copyout_ms += ms; }
   st.depth_bytes += st.depth_rows_bytes;
   st.n_groups = n_groups;
   st.n_launches = launches;

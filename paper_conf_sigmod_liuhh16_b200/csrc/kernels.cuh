@@ -84,6 +84,7 @@ struct HubChunk {
 // Per group per level counters (device).  dir: 0 = level not run, 1 = TD, 2 = BU.
 struct LevelStat {
   unsigned long long jfq, fq, proc, insp, writes, newp, nf;
+  unsigned long long gath;  // neighbour status words actually gathered (BU frontier hits, TD pre-checks)
   uint32_t dir;
   uint32_t flags;    // bit 0: the depth kernel skips this level's snapshot (late list +
                      // fix-up); bit 1: the level's commit was sparse
@@ -105,6 +106,15 @@ struct GroupCtrl {
   // td_bits = the active instances expanded top-down in the next level when dir == BU
   T td_bits;
   uint32_t sparse;  // the last commit was sparse (no bottom-up queue: the next level is TD)
+  // the next expand marks the 32-vertex chunks it writes (for a sparse commit): only for a
+  // top-down level whose frontier edge count m_f could leave few writes (m_f <= 2 nva); a
+  // heavy level (level 2 of a hub-sharing group: m_f ~ 10^8) is never sparse, and a byte
+  // store per RED.OR would add a third write request to every update
+  uint32_t td_mark;
+  // the next bottom-up expand probes the frontier bitmap before gathering (Policy::bu_probe):
+  // worth it when the frontier (vertices with new bits) is a small part of the graph, so
+  // most neighbours are not in it; on a dense frontier the probe only adds latency
+  uint32_t bu_probe;
   // levels whose snapshot the depth kernel does not read (bit l): level 0 (the sources,
   // written by late_fix_kernel from the source list) and every sparse-committed level,
   // whose few new vertices went to the late list instead
@@ -123,6 +133,7 @@ struct Policy {
   uint32_t split, split_mod;  // IBFS_SPLIT_*
   float split_div;
   uint32_t max_depth;  // k-hop cap (0 = unbounded)
+  uint32_t bu_probe;   // frontier-bitmap probes in BU: 0 never, 1 sparse frontiers (default), 2 always
   uint8_t sched[MAXL];  // 0 TD / 1 BU for level l at index l-1
 };
 
@@ -148,6 +159,12 @@ struct BatchArgs {
   int gcap;      // groups allocated per slot
   uint32_t *tdq, *buq;  // [gcap][nva] queues
   uint8_t *dirty;       // [gcap][nchunk32] 32-vertex chunk of S_l written by a top-down RED.OR
+  // [gcap][nchunk32] frontier bitmap of the running level: bit v%32 of word v/32 = (S_l-1[v]
+  // != 0), written by the commit of level l-1 (the init for level 1).  Bottom-up needs a
+  // neighbour's word only when the neighbour is in the frontier (Lemma: visited[w] & T[f]
+  // = S_l-1[w] & T[f]), so the bitmap -- nva/8 bytes per group, L2-resident --
+  // filters the random status gathers.
+  uint32_t *fbits;
   unsigned long long *late;  // [gcap][late_cap] (level << 32 | v) new vertices of sparse commits
   uint32_t *late_n;          // [gcap] appended entries (may exceed late_cap: then no more skips)
   uint32_t late_cap;
@@ -313,11 +330,12 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
   __shared__ uint32_t s_src[W];
   __shared__ uint32_t s_distinct;
   __shared__ T s_act;
+  __shared__ unsigned long long s_msrc;
   const int g = blockIdx.x;
   const int rows = group_rows(a, g);
   LevelStat *ls = a.lstat + (size_t)g * MAXL;
   for (int l = threadIdx.x; l < MAXL; l += blockDim.x) ls[l] = LevelStat{};
-  if (threadIdx.x == 0) { s_distinct = 0; s_act = wzero_value<T>(); }
+  if (threadIdx.x == 0) { s_distinct = 0; s_act = wzero_value<T>(); s_msrc = 0; }
   for (int j = threadIdx.x; j < rows; j += blockDim.x) s_src[j] = a.src[(size_t)g * W + j];
   __syncthreads();
   for (int j = threadIdx.x; j < rows; j += blockDim.x) {
@@ -325,7 +343,11 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     for (int i = 0; i < j; ++i)
       if (s_src[i] == s_src[j]) { first = false; break; }
     if (first) atomicAdd(&s_distinct, 1u);
-    if (a.csrc[(size_t)g * W + j] != NO_VERTEX) set_bit_atomic(&s_act, j);
+    const uint32_t cs = a.csrc[(size_t)g * W + j];
+    if (cs != NO_VERTEX) {
+      set_bit_atomic(&s_act, j);
+      atomicAdd(&s_msrc, (unsigned long long)__ldg(a.deg + cs));
+    }
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -338,6 +360,8 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
       for (int k = 0; k < NQ; ++k) c.qlen[p][k] = 0;
     c.dir = first_dir;
     c.td_filter = 0;
+    c.td_mark = s_msrc <= 2ull * a.nva ? 1u : 0u;  // level 1's frontier edges: the sources' rows
+    c.bu_probe = a.pol.bu_probe != 0 ? 1u : 0u;    // level 1's frontier: the sources
     const bool done = rows == 0 || wzero(s_act);
     c.done = done ? 1u : 0u;
     c.arrive = 0;
@@ -394,7 +418,10 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
       st(vis + v, z);
       st(s0 + v, z);
       st(s1 + v, z);
-      if ((v & 31) == 0) a.dirty[(size_t)g * a.nchunk32 + (v >> 5)] = 0;
+      if ((v & 31) == 0) {
+        a.dirty[(size_t)g * a.nchunk32 + (v >> 5)] = 0;
+        a.fbits[(size_t)g * a.nchunk32 + (v >> 5)] = 0u;
+      }
     }
     if (first_dir) {
       const uint32_t d = in ? __ldg(a.rdeg + v) : 0u;  // bottom-up reads in-edge rows
@@ -427,6 +454,7 @@ __global__ void init_sources_kernel(BatchArgs<T> a, uint32_t first_dir) {
       s = s_src[j];
       set_bit_atomic(vis + s, j);
       set_bit_atomic(f + s, j);
+      atomicOr(a.fbits + (size_t)g * a.nchunk32 + (s >> 5), 1u << (s & 31));
       first = true;
       for (int i = 0; i < j; ++i)
         if (s_src[i] == s) { first = false; break; }
@@ -446,7 +474,7 @@ struct ExpandSmem {  // static part
   uint32_t item;
   uint32_t flag;
   uint32_t pre[3 * MAX_G * 2 + 1];   // item prefix over (phase, group, direction)
-  unsigned long long acc[MAX_G][5];  // jfq, fq, proc, insp, writes
+  unsigned long long acc[MAX_G][6];  // jfq, fq, proc, insp, writes, gath
 };
 
 // Dynamic part: the CTA-local copy of one work item's queue entries.
@@ -511,18 +539,20 @@ __device__ __forceinline__ uint32_t lbs_search(const uint32_t *s, uint32_t n, ui
 }
 
 __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq, uint32_t fq,
-                                             uint32_t proc, uint32_t insp, uint32_t writes) {
+                                             uint32_t proc, uint32_t insp, uint32_t writes, uint32_t gath) {
   jfq = __reduce_add_sync(FULL, jfq);
   fq = __reduce_add_sync(FULL, fq);
   proc = __reduce_add_sync(FULL, proc);
   insp = __reduce_add_sync(FULL, insp);
   writes = __reduce_add_sync(FULL, writes);
+  gath = __reduce_add_sync(FULL, gath);
   if ((threadIdx.x & 31) == 0) {
     if (jfq) atomicAdd(&sm.acc[g][0], (unsigned long long)jfq);
     if (fq) atomicAdd(&sm.acc[g][1], (unsigned long long)fq);
     if (proc) atomicAdd(&sm.acc[g][2], (unsigned long long)proc);
     if (insp) atomicAdd(&sm.acc[g][3], (unsigned long long)insp);
     if (writes) atomicAdd(&sm.acc[g][4], (unsigned long long)writes);
+    if (gath) atomicAdd(&sm.acc[g][5], (unsigned long long)gath);
   }
 }
 
@@ -534,14 +564,14 @@ __device__ __forceinline__ void flush_counts(ExpandSmem &sm, int g, uint32_t jfq
 // BU level); entries whose frontier word has none of them sweep no edges.
 template <typename T>
 __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq, int g, int cls,
-                        uint32_t i0, uint32_t i1, int level, bool filt, T fmask) {
+                        uint32_t i0, uint32_t i1, int level, bool filt, T fmask, bool mark) {
   const int tid = threadIdx.x;
   const T *F = frontier_buf(a, g, level);
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
   const uint32_t *q = queue_of(a, g, cls);
   const uint32_t qn = i1 - i0;
-  uint32_t insp = 0, writes = 0;
+  uint32_t insp = 0, writes = 0, gath = 0;
   for (uint32_t i = tid; i < qn; i += BLOCK) {
     const uint32_t v = queue_at(a, q, cls, i0 + i);
     const T f = wand(ldg(F + v), fmask);
@@ -570,12 +600,17 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
     for (int u = 0; u < U; ++u) {
       if (w[u] != 0xffffffffu) {
         insp++;
+        gath += filt ? 1u : 0u;
         const T b = filt ? wandn(fw[u], ldg(vis + w[u])) : fw[u];
-        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u]); }
+        if (!wzero(b)) {
+          red_or(N + w[u], b);
+          writes++;
+          if (mark) mark_dirty(a, g, w[u]);
+        }
       }
     }
   }
-  flush_counts(sm, g, 0u, 0u, tid == 0 ? qn : 0u, insp, writes);
+  flush_counts(sm, g, 0u, 0u, tid == 0 ? qn : 0u, insp, writes, gath);
 }
 
 // Bottom-up item: entries [i0, i1) of a BU queue class.
@@ -599,15 +634,17 @@ template <typename T>
 // split level expands top-down instead (excluded from T; N[f] is then shared with the
 // top-down part, so the result is ORed in rather than stored).
 __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq, int g, int cls,
-                        uint32_t i0, uint32_t i1, int level, T active, T td_bits) {
+                        uint32_t i0, uint32_t i1, int level, T active, T td_bits, bool probe) {
   constexpr int QW = QL / NWARP;  // ring entries per warp (128)
   static_assert(sizeof(BuRing<T>) <= sizeof(TileQueue<T>), "BU ring must fit the item storage");
   BuRing<T> &bq = *reinterpret_cast<BuRing<T> *>(&tq);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
+  const T *F = frontier_buf(a, g, level);                 // S_l-1: the neighbours' new bits
+  const uint32_t *fb = a.fbits + (size_t)g * a.nchunk32;  // its nonzero bitmap
   const uint32_t *q = queue_of(a, g, cls);
-  uint32_t jfq = 0, fq = 0, proc = 0, insp = 0, writes = 0;
+  uint32_t jfq = 0, fq = 0, proc = 0, insp = 0, writes = 0, gath = 0;
   const bool split = !wzero(td_bits);
   if (tid == 0) sm.cnt[0] = i0;
   __syncthreads();
@@ -618,7 +655,10 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
   uint32_t v = 0, d = 0, k = 0;
   unsigned long long s0 = 0;
   T tg = wzero_value<T>(), acc = wzero_value<T>();
-  uint32_t wn[BU_U];  // adjacency entries of the lane's next step (prefetched)
+  // software pipeline over a row, BU_U neighbours per step: the step's ids and their
+  // frontier-bitmap words are in (wn, mn); the next step's ids in wn2 (prefetched); the
+  // bitmap words of step s + 1 are loaded during step s
+  uint32_t wn[BU_U], mn[BU_U], wn2[BU_U];
   // refill pipeline: the loads for the next 32 queue entries are issued one round early
   uint32_t c_next = 0, x_next = 0, dx_next = 0;
   T tx_next = wzero_value<T>();
@@ -676,6 +716,13 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
         proc++;
 #pragma unroll
         for (int u = 0; u < BU_U; ++u) wn[u] = ((uint32_t)u < d) ? __ldg(a.radj + s0 + u) : 0xffffffffu;
+#pragma unroll
+        for (int u = 0; u < BU_U; ++u) wn2[u] = ((uint32_t)(BU_U + u) < d) ? __ldg(a.radj + s0 + BU_U + u) : 0xffffffffu;
+        // the first step gathers without the bitmap probe: most vertices stop within their
+        // first neighbours (hub-first rows, frontier hubs), and a probe there would put an
+        // L2 round trip on every vertex's critical path
+#pragma unroll
+        for (int u = 0; u < BU_U; ++u) mn[u] = 0xffffffffu;
       }
     }
     head += min((uint32_t)__popc(idle), avail);
@@ -686,18 +733,26 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       continue;
     }
     if (has) {
-      uint32_t w[BU_U];
-#pragma unroll
-      for (int u = 0; u < BU_U; ++u) w[u] = wn[u];
+      // neighbour w contributes visited[w] & T = S_l-1[w] & T (a bit of T visited at w
+      // before level l-1 would have reached f already): gather S_l-1[w] only when w is in
+      // the frontier bitmap
       T x[BU_U];
 #pragma unroll
-      for (int u = 0; u < BU_U; ++u) x[u] = w[u] != 0xffffffffu ? ldg(vis + w[u]) : wzero_value<T>();
+      for (int u = 0; u < BU_U; ++u) {
+        const bool hit = wn[u] != 0xffffffffu && ((mn[u] >> (wn[u] & 31)) & 1u);
+        x[u] = hit ? ldg(F + wn[u]) : wzero_value<T>();
+        gath += hit ? 1u : 0u;
+        insp += wn[u] != 0xffffffffu ? 1u : 0u;
+      }
       k += BU_U;
 #pragma unroll
-      for (int u = 0; u < BU_U; ++u) wn[u] = (k + u < d) ? __ldg(a.radj + s0 + k + u) : 0xffffffffu;
+      for (int u = 0; u < BU_U; ++u) wn[u] = wn2[u];
 #pragma unroll
-      for (int u = 0; u < BU_U; ++u)
-        if (w[u] != 0xffffffffu) { acc = wor(acc, wand(x[u], tg)); insp++; }
+      for (int u = 0; u < BU_U; ++u) mn[u] = (probe && wn[u] != 0xffffffffu) ? __ldg(fb + (wn[u] >> 5)) : 0xffffffffu;
+#pragma unroll
+      for (int u = 0; u < BU_U; ++u) wn2[u] = (k + BU_U + u < d) ? __ldg(a.radj + s0 + k + BU_U + u) : 0xffffffffu;
+#pragma unroll
+      for (int u = 0; u < BU_U; ++u) acc = wor(acc, wand(x[u], tg));
       if (weq(acc, tg) || k >= d) {
         if (!wzero(acc)) {
           if (split) red_or(N + v, acc); else st(N + v, acc);
@@ -707,20 +762,20 @@ __device__ void item_bu(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       }
     }
   }
-  flush_counts(sm, g, jfq, fq, proc, insp, writes);
+  flush_counts(sm, g, jfq, fq, proc, insp, writes, gath);
 }
 
 // Hub chunk, top-down: CHUNK edges of one hub's row swept by the whole CTA.
 template <typename T>
 __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubChunk c, int level, bool filt,
-                       T fmask) {
+                       T fmask, bool mark) {
   const int tid = threadIdx.x;
   const T *F = frontier_buf(a, g, level);
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
   const T f = wand(ldg(F + c.v), fmask);
   if (wzero(f)) return;
-  uint32_t insp = 0, writes = 0;
+  uint32_t insp = 0, writes = 0, gath = 0;
   constexpr int U = 8;
   for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
     uint32_t w[U];
@@ -733,13 +788,18 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
     for (int u = 0; u < U; ++u) {
       if (w[u] != 0xffffffffu) {
         insp++;
+        gath += filt ? 1u : 0u;
         const T b = filt ? wandn(f, ldg(vis + w[u])) : f;
-        if (!wzero(b)) { red_or(N + w[u], b); writes++; mark_dirty(a, g, w[u]); }
+        if (!wzero(b)) {
+          red_or(N + w[u], b);
+          writes++;
+          if (mark) mark_dirty(a, g, w[u]);
+        }
       }
     }
   }
   const bool first = c.first && tid == 0;
-  flush_counts(sm, g, 0u, 0u, first ? 1u : 0u, insp, writes);
+  flush_counts(sm, g, 0u, 0u, first ? 1u : 0u, insp, writes, gath);
 }
 
 // Hub chunk, bottom-up: the CTA ORs a chunk of the hub's neighbours in waves, with a
@@ -747,33 +807,47 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
 // already found (atomically accumulated in N[hub]).
 template <typename T>
 __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, const HubChunk c,
-                       int level, T active, T td_bits) {
+                       int level, T active, T td_bits, bool probe) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   T *N = next_buf(a, g, level);
   const T *vis = a.visited + (size_t)g * a.gstride;
+  const T *F = frontier_buf(a, g, level);
+  const uint32_t *fb = a.fbits + (size_t)g * a.nchunk32;
   const T tfull = wandn(active, ldg(vis + c.v));
   const T tg = wandn(tfull, td_bits);
   const bool first = c.first && tid == 0;
   const bool cnt = first && level > 1 && !wzero(tfull);  // level 1: closed form (init)
   if (wzero(tg)) {
-    flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tfull) : 0u, 0u, 0u, 0u);
+    flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tfull) : 0u, 0u, 0u, 0u, 0u);
     return;
   }
   if (tid == 0) sm.flag = weq(wand(ldv(N + c.v), tg), tg) ? 1u : 0u;
   __syncthreads();
-  uint32_t insp = 0, writes = 0;
+  uint32_t insp = 0, writes = 0, gath = 0;
   T acc = wzero_value<T>();
   if (!sm.flag) {
     constexpr int U = 4;
     for (unsigned long long e0 = c.e0; e0 < c.e1; e0 += BLOCK * U) {
       T x = wzero_value<T>();
+      uint32_t w[U], m[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const unsigned long long e = e0 + u * BLOCK + tid;
-        if (e < c.e1) {
-          const uint32_t w = __ldg(a.radj + e);
-          x = wor(x, wand(ldg(vis + w), tg));
+        w[u] = e < c.e1 ? __ldg(a.radj + e) : 0xffffffffu;
+      }
+      // the first wave (the row's highest-degree neighbours) gathers directly; later waves
+      // probe the frontier bitmap first
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        m[u] = (e0 == c.e0 || !probe) ? 0xffffffffu : (w[u] != 0xffffffffu ? __ldg(fb + (w[u] >> 5)) : 0u);
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (w[u] != 0xffffffffu) {
           insp++;
+          if ((m[u] >> (w[u] & 31)) & 1u) {  // frontier neighbour: S_l-1[w] & T (see item_bu)
+            x = wor(x, wand(ldg(F + w[u]), tg));
+            gath++;
+          }
         }
       }
       x = warp_or(x);
@@ -787,7 +861,7 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
     }
     if (tid == 0 && !wzero(acc)) { red_or(N + c.v, acc); writes++; }
   }
-  flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tfull) : 0u, first ? 1u : 0u, insp, writes);
+  flush_counts(sm, g, cnt ? 1u : 0u, cnt ? (uint32_t)wpopc(tfull) : 0u, first ? 1u : 0u, insp, writes, gath);
 }
 
 // Expand phase of level `level` for all groups of a batch.  Work items, pulled by CTAs
@@ -799,7 +873,7 @@ __device__ void hub_bu(const BatchArgs<T> &a, ExpandSmem &sm, T *s_red, int g, c
 template <typename T>
 __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T *s_red, TileQueue<T> &tq) {
   const int tid = threadIdx.x;
-  for (int i = tid; i < a.G * 5; i += BLOCK) sm.acc[i / 5][i % 5] = 0ull;
+  for (int i = tid; i < a.G * 6; i += BLOCK) sm.acc[i / 6][i % 6] = 0ull;
   const int par = (level - 1) & 1;  // queues were produced by commit l-1 (or init)
   const int nslot = 3 * a.G * 2;
   for (int i = tid; i < nslot; i += BLOCK) {  // items of slot (phase, group, direction)
@@ -859,11 +933,13 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     const T td_bits = bu_level ? ldcg_w(&c->td_bits) : wzero_value<T>();
     const T all = wnot(wzero_value<T>());
     const bool filt = ldcg(&c->td_filter) != 0;
+    const bool mark = !bu_level && ldcg(&c->td_mark) != 0;
+    const bool probe = ldcg(&c->bu_probe) != 0;
     if (ph == 0) {
       const uint32_t ci = a.chq[((size_t)g * 2 + d) * a.chq_stride + k];
       const HubChunk hc = d ? a.rchunks[ci] : a.chunks[ci];
-      if (d == 0) hub_td<T>(a, sm, g, hc, level, filt, bu_level ? td_bits : all);
-      else hub_bu<T>(a, sm, s_red, g, hc, level, ldcg_w(&c->active), td_bits);
+      if (d == 0) hub_td<T>(a, sm, g, hc, level, filt, bu_level ? td_bits : all, mark);
+      else hub_bu<T>(a, sm, s_red, g, hc, level, ldcg_w(&c->active), td_bits, probe);
       continue;
     }
     const bool heavy = ph == 1;
@@ -871,8 +947,8 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     const uint32_t qlen = ldcg(c->qlen[par] + cls);
     const uint32_t per = d ? (heavy ? QBH : QL) : (heavy ? QH : QL);
     const uint32_t i0 = k * per, i1 = min(qlen, i0 + per);
-    if (d == 0) item_td<T>(a, sm, tq, g, cls, i0, i1, level, filt, bu_level ? td_bits : all);
-    else item_bu<T>(a, sm, tq, g, cls, i0, i1, level, ldcg_w(&c->active), td_bits);
+    if (d == 0) item_td<T>(a, sm, tq, g, cls, i0, i1, level, filt, bu_level ? td_bits : all, mark);
+    else item_bu<T>(a, sm, tq, g, cls, i0, i1, level, ldcg_w(&c->active), td_bits, probe);
   }
   __syncthreads();
   for (int i = tid; i < a.G; i += BLOCK) {
@@ -882,6 +958,7 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     if (sm.acc[i][2]) atomicAdd(&ls->proc, sm.acc[i][2]);
     if (sm.acc[i][3]) atomicAdd(&ls->insp, sm.acc[i][3]);
     if (sm.acc[i][4]) atomicAdd(&ls->writes, sm.acc[i][4]);
+    if (sm.acc[i][5]) atomicAdd(&ls->gath, sm.acc[i][5]);
   }
 }
 
@@ -952,7 +1029,7 @@ constexpr int SAMPLE = SAMPLE_TILES * CVT;
 // every CTA from state fixed before this launch.
 template <typename T>
 __device__ __forceinline__ bool commit_sparse(const BatchArgs<T> &a, const GroupCtrl<T> *c, int lc) {
-  if (c->dir != 0) return false;
+  if (c->dir != 0 || !c->td_mark) return false;
   // every write marks at most one chunk: the level's write count bounds the marked ones
   if (a.lstat[(size_t)(c - a.ctrl) * MAXL + lc].writes * 4ull > (unsigned long long)a.nchunk32) return false;
   const uint32_t next = (uint32_t)lc + 1;
@@ -1031,6 +1108,12 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
     }
     const bool nz = !wzero(n[k]);
     if (nz) st(vis + v, wor(vv[k], n[k]));
+    {  // frontier bitmap of level lc + 1 (read by its bottom-up gathers); every chunk is
+       // rewritten, sparse commits included (their untouched chunks hold no new bit)
+      const uint32_t fball = __ballot_sync(FULL, nz);
+      const size_t ch = (base + (size_t)k * BLOCK + (size_t)(warp * 32)) >> 5;
+      if (lane == 0 && ch < a.nchunk32) a.fbits[(size_t)g * a.nchunk32 + ch] = fball;
+    }
     if (sparse) {  // block-uniform: the new vertices of a sparse level go to the late list
       const uint32_t lb = __ballot_sync(FULL, nz);
       if (lb) {
@@ -1225,6 +1308,8 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     c->n_f = c->m_f = c->newp = 0;
     c->dir = bu ? 1u : 0u;
     c->td_bits = tdb;
+    c->td_mark = (!bu && (double)m_f <= 2.0 * (double)a.nva) ? 1u : 0u;
+    c->bu_probe = a.pol.bu_probe == 2 || (a.pol.bu_probe == 1 && n_f * 8ull < (unsigned long long)a.nva) ? 1u : 0u;
     // top-down pre-check of visited[w] only once a fair share of the (vertex, active
     // instance) pairs is visited; before that nearly every OR is new and the gather is
     // wasted (the commit masks what an unfiltered OR set twice)
@@ -1703,6 +1788,259 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DEPTH_MINB)
         }
       }
     }
+  }
+}
+
+// ---- depth rows, TMA-store variant (the default when the rows allow it) ----
+// The store pattern decides this kernel's speed: 4-byte streaming stores that put 32 bytes
+// in each of 4 rows per warp instruction top out at ~1.7 TB/s on B200 (profiles/r02/
+// randbench.json "st32_rows_gbs"; every 32-byte sector is its own L2 write request), while
+// whole 128-byte lines stream at ~6.2 TB/s.  So the rows of a 128-column x W-row tile are
+// assembled row-major in shared memory and leave as ONE 2-D bulk tensor store (TMA,
+// cp.async.bulk.tensor): full lines, no store instructions on the SM, no lane transposes.
+//   fill    the tile's buffer = 0xff (-1: isolated columns, unreached instances);
+//   phase A as in depth_kernel (thread = dense slot x instance part, SIMD-within-register
+//           accumulation of l + 1 over the loaded snapshot levels), then each thread writes
+//           its column's bytes straight into their rows (byte stores; a warp = 32 columns
+//           of one row: one shared-memory wavefront);
+//   store   fence.proxy.async, barrier, one thread issues the tensor store; the buffer is
+//           reused two tiles later, after cp.async.bulk.wait_group.read.
+// Only for a batch's first (complete) flush; ring-slot re-flushes and rows that break the
+// tensor map's alignment rules use depth_kernel.
+#ifndef IBFS_DTMA_DLB
+#define IBFS_DTMA_DLB 5
+#endif
+#ifndef IBFS_DTMA_NS
+#define IBFS_DTMA_NS 4
+#endif
+#ifndef IBFS_DTMA_MINB
+#define IBFS_DTMA_MINB 3
+#endif
+constexpr int DLB2 = IBFS_DTMA_DLB;  // loaded snapshot levels per pipeline stage
+constexpr int DNS2 = IBFS_DTMA_NS;   // pipeline stages
+constexpr int DMAXL = 128;           // levels a flush can cover (depths <= 127)
+
+template <typename T>
+struct DepthTmaLayout {
+  static constexpr int W = WordBits<T>::value;
+  static constexpr size_t TILE = (size_t)DV * W;                     // one row-major output tile
+  static constexpr size_t SROW = (size_t)DV * sizeof(T) + 16;
+  static constexpr size_t STAGE = DHDR + DLB2 * SROW;
+  static constexpr size_t BYTES = 128 + 2 * TILE + DNS2 * STAGE;
+  static_assert(TILE % 128 == 0 && STAGE % 16 == 0, "tiles stay 128-byte aligned");
+  static_assert(DLB2 <= 16, "stage header holds 16 level bytes");
+};
+
+template <typename T>
+constexpr size_t depth_tma_smem_bytes() {
+  return DepthTmaLayout<T>::BYTES;
+}
+
+__device__ __forceinline__ void sts8(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "r"(v));
+}
+
+// Stage header (DHDR bytes): [0] k (non-isolated columns of the tile), [4] byte offset of
+// the runs, [8] c0, [12] nl (loaded levels in this stage), [16 .. 16 + DLB2) the level + 1 of
+// each slot, [32 .. 32 + DV) dense slot -> column.  A tile takes ceil(loaded levels / DLB2)
+// stages (at least one, for its header); only loaded levels occupy slots.
+template <typename T>
+__global__ void __launch_bounds__(DTHREADS + 32, IBFS_DTMA_MINB)
+    depth_tma_kernel(const __grid_constant__ CUtensorMap tmap, BatchArgs<T> a, int l0, int l1) {
+  using L = DepthTmaLayout<T>;
+  constexpr int W = WordBits<T>::value;
+  constexpr int PB = W / 4;   // instances per part
+  constexpr int PQ = PB / 4;  // byte registers per part
+  extern __shared__ unsigned char dsm_raw[];
+  const uint32_t sbase = (smem_u32(dsm_raw) + 127u) & ~127u;
+  const uint32_t outb = sbase;  // [2][W][DV] row-major output tiles
+  const uint32_t stage_base = sbase + 2 * (uint32_t)L::TILE;
+  __shared__ __align__(8) unsigned long long s_full[DNS2], s_empty[DNS2];
+  __shared__ const T *s_run[DMAXL];  // snapshot array of each loaded level, in level order
+  __shared__ uint8_t s_inc[DMAXL];   // its level + 1
+  __shared__ int s_nload;
+  const int g = blockIdx.y;
+  const int rows = group_rows(a, g);
+  if (rows == 0) return;
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  const GroupCtrl<T> *c = a.ctrl + g;
+  const int last = min((int)c->last_level, min(l1, 127));
+  const size_t nvv = a.nv;
+  const size_t ntiles = (nvv + DV - 1) / DV;
+  if (t == 0) {
+    // the loaded levels (skipped ones come from the late list / source list): their ring
+    // slot arrays, computed once
+    const unsigned long long sk0 = c->skip_lv[0], sk1 = c->skip_lv[1];
+    int n = 0;
+    for (int l = l0; l <= last; ++l) {
+      const bool sk = ((l < 64 ? sk0 >> l : sk1 >> (l - 64)) & 1ull) != 0;
+      if (sk) continue;
+      s_run[n] = snap(a, g, l);
+      s_inc[n] = (uint8_t)(l + 1);
+      ++n;
+    }
+    s_nload = n;
+    for (int k = 0; k < DNS2; ++k) {
+      mbar_init(&s_full[k], 32);
+      mbar_init(&s_empty[k], DCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const int nload = s_nload;
+  const int nbat = nload > 0 ? (nload + DLB2 - 1) / DLB2 : 1;  // >= 1 stage per tile (its header)
+  const size_t my_tiles = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+  const size_t njobs = my_tiles * (size_t)nbat;
+  const uint32_t full0 = smem_u32(&s_full[0]), empty0 = smem_u32(&s_empty[0]);
+  if (warp == DCW) {
+    // ---- producer: job jb = (tile jb / nbat of this CTA, stage batch jb % nbat)
+    int st = 0;
+    uint32_t ph = 0;
+    for (size_t jb = 0; jb < njobs; ++jb) {
+      const int b = (int)(jb % nbat);
+      const size_t tix = blockIdx.x + (jb / nbat) * gridDim.x;
+      const uint32_t c0 = __ldg(a.tbase + tix), k = __ldg(a.tbase + tix + 1) - c0;
+      const int s0 = b * DLB2, nl = max(0, min(DLB2, nload - s0));
+      uint32_t off = 0, size = 0;
+      if (k && nl) {
+        const uintptr_t src0 = (uintptr_t)(s_run[s0] + c0);
+        off = (uint32_t)(src0 & 15u);
+        size = (uint32_t)((off + (size_t)k * sizeof(T) + 15) & ~(size_t)15);
+      }
+      if (jb >= (size_t)DNS2) mbar_wait(reinterpret_cast<unsigned long long *>(&s_empty[st]), ph ^ 1u);
+      const uint32_t sb = stage_base + (uint32_t)(st * L::STAGE);
+      if (b == 0) {  // the tile's dense slot -> column table (read by the consumers at b == 0)
+        const uint4 nzw = __ldg(reinterpret_cast<const uint4 *>(a.nzbits) + tix);
+        const uint32_t wv = lane < 8 ? nzw.x : lane < 16 ? nzw.y : lane < 24 ? nzw.z : nzw.w;
+        const uint32_t nib = (wv >> (4 * (lane & 7))) & 0xFu;
+        const uint32_t cnt = __popc(nib);
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const uint32_t y = __shfl_up_sync(FULL, incl, d);
+          if (lane >= d) incl += y;
+        }
+        uint32_t pos = incl - cnt;
+#pragma unroll
+        for (int cc = 0; cc < 4; ++cc)
+          if ((nib >> cc) & 1u) {
+            asm volatile("st.shared.u8 [%0], %1;" ::"r"(sb + 32 + pos), "h"((unsigned short)(4 * lane + cc)));
+            ++pos;
+          }
+      }
+      if (lane < nl) sts8(sb + 16 + lane, s_inc[s0 + lane]);
+      if (lane == 0) sts128(sb, k, off, c0, (uint32_t)nl);
+      const uint32_t total = size * (uint32_t)nl;
+      if (lane == 0) mbar_arrive_expect_tx(&s_full[st], total); else mbar_arrive(&s_full[st]);
+      if (lane < nl && total) {
+        const unsigned char *src = reinterpret_cast<const unsigned char *>(s_run[s0 + lane] + c0) - off;
+        bulk_g2s(sb + DHDR + (uint32_t)(lane * L::SROW), src, size, &s_full[st]);
+      }
+      if (++st == DNS2) { st = 0; ph ^= 1u; }
+    }
+  } else {
+    // ---- consumers
+    const int part = t / DSLOTS, dslot = t % DSLOTS;
+    int st = 0;
+    uint32_t ph = 0;
+    int buf = 0;
+    for (size_t tix = blockIdx.x; tix < ntiles; tix += gridDim.x, buf ^= 1) {
+      const uint32_t ob = outb + (uint32_t)(buf * L::TILE);
+      // the tensor store issued from this buffer two tiles ago has finished reading it
+      if (t == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+      consumers_sync();
+#pragma unroll
+      for (uint32_t j = 0; j < (uint32_t)(L::TILE / 16 / DTHREADS); ++j)
+        sts128(ob + 16 * ((uint32_t)t + j * DTHREADS), 0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu);
+      uint32_t acc[2][PQ];
+#pragma unroll
+      for (int r = 0; r < 2; ++r)
+#pragma unroll
+        for (int q = 0; q < PQ; ++q) acc[r][q] = 0;
+      uint32_t reached[2] = {0u, 0u};
+      uint32_t k = 0, dcol[2] = {0u, 0u};
+      for (int b = 0; b < nbat; ++b) {
+        asm volatile(
+            "{\n .reg .pred p;\n WAIT_%=:\n"
+            " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
+            " @!p bra WAIT_%=;\n}\n" ::"r"(full0 + 8u * (uint32_t)st),
+            "r"(ph), "r"(1000000u)
+            : "memory");
+        const uint32_t sb = stage_base + (uint32_t)(st * L::STAGE);
+        const uint4 hdr = lds128(sb);  // k, off, c0, nl
+        if (b == 0) {
+          k = hdr.x;
+#pragma unroll
+          for (int r = 0; r < 2; ++r) {
+            const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
+            if (i < k) dcol[r] = lds8(sb + 32 + i);
+          }
+        }
+        const uint32_t nl = hdr.w;
+        const uint4 incs = lds128(sb + 16);
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+          const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
+          if (i < k) {
+            const uint32_t p = sb + DHDR + hdr.y + i * (uint32_t)sizeof(T) + (uint32_t)(part * PB / 8);
+#pragma unroll
+            for (int u = 0; u < DLB2; ++u) {
+              if ((uint32_t)u >= nl) break;
+              const uint32_t hb = lds_part<PB>(p + (uint32_t)(u * L::SROW)) & ~reached[r];
+              if (!hb) continue;
+              const uint32_t iw = u < 4 ? incs.x : u < 8 ? incs.y : u < 12 ? incs.z : incs.w;
+              const uint32_t inc = (iw >> (8 * (u & 3))) & 0xffu;
+              if (reached[r] == 0u && hb == (PB == 32 ? 0xffffffffu : ((1u << PB) - 1u))) {
+#pragma unroll
+                for (int q = 0; q < PQ; ++q) acc[r][q] = inc * 0x01010101u;
+              } else if (PB == 32) {
+                // byte b of word q holds instance q + 8b (not 4q + b): its bit is (hb >> q)
+                // bit 8b, so the spread is one shift and one mask
+#pragma unroll
+                for (int q = 0; q < PQ; ++q) acc[r][q] += ((hb >> q) & 0x01010101u) * inc;
+              } else {
+#pragma unroll
+                for (int q = 0; q < PQ; ++q) acc[r][q] += spread4((hb >> (4 * q)) & 0xFu) * inc;
+              }
+              reached[r] |= hb;
+            }
+          }
+        }
+        __syncwarp();
+        if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(empty0 + 8u * (uint32_t)st) : "memory");
+        if (++st == DNS2) { st = 0; ph ^= 1u; }
+      }
+      consumers_sync();  // the 0xff fill is complete
+      // the column's bytes into their rows (a warp writes 32 columns of one row per store):
+      // byte bb of word q is instance q + 8 bb (W = 128) or 4q + bb (W = 32, 64) of the part
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const uint32_t i = (uint32_t)(dslot + DSLOTS * r);
+        if (i < k) {
+          const uint32_t base = ob + (uint32_t)(part * PB) * DV + dcol[r];
+#pragma unroll
+          for (int q = 0; q < PQ; ++q) {
+            const uint32_t w = __vsub4(acc[r][q], 0x01010101u);  // l + 1 -> l, 0 -> 0xff (-1)
+#pragma unroll
+            for (int bb = 0; bb < 4; ++bb) {
+              const uint32_t inst = PB == 32 ? (uint32_t)(q + 8 * bb) : (uint32_t)(4 * q + bb);
+              sts8(base + inst * DV, w >> (8 * bb));
+            }
+          }
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      consumers_sync();
+      if (t == 0) {
+        const int c0i = (int)(tix * DV), r0i = g * W;
+        asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                         reinterpret_cast<uint64_t>(&tmap)),
+                     "r"(ob), "r"(c0i), "r"(r0i)
+                     : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
+    }
+    if (t == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
 }
 

@@ -95,6 +95,7 @@ class RunStats:
     ms_ms: float
     ms_launches: int
     level_launches_live: int
+    words_gathered: int
     per_source_m: np.ndarray | None = None
     per_source_digest: np.ndarray | None = None
     per_level: list = field(default_factory=list)

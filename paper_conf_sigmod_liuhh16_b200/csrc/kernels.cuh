@@ -932,7 +932,10 @@ __device__ void expand_phase(const BatchArgs<T> &a, int level, ExpandSmem &sm, T
     const bool bu_level = ldcg(&c->dir) == 1;
     const T td_bits = bu_level ? ldcg_w(&c->td_bits) : wzero_value<T>();
     const T all = wnot(wzero_value<T>());
-    const bool filt = ldcg(&c->td_filter) != 0;
+    // the top-down part of a split bottom-up level expands instances that are still early
+    // in their traversal (most targets unvisited for them): no visited pre-check gather,
+    // the RED.ORs go out directly (the commit masks bits that were already visited)
+    const bool filt = !bu_level && ldcg(&c->td_filter) != 0;
     const bool mark = !bu_level && ldcg(&c->td_mark) != 0;
     const bool probe = ldcg(&c->bu_probe) != 0;
     if (ph == 0) {
@@ -1038,6 +1041,16 @@ __device__ __forceinline__ bool commit_sparse(const BatchArgs<T> &a, const Group
     case 2: return next < a.pol.bu_from;
     default: return next - 1 < a.pol.sched_len ? a.pol.sched[next - 1] == 0 : true;
   }
+}
+
+template <typename T>
+__device__ __forceinline__ void prefetch_commit_tile(const BatchArgs<T> &a, int g, int lc, size_t base) {
+  const uint32_t nvt = (uint32_t)min((size_t)CTILE, (size_t)a.nva - base);
+  const uint32_t wb = (nvt * (uint32_t)sizeof(T) + 15u) & ~15u, db = (nvt * 4u + 15u) & ~15u;
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(snap(a, g, lc) + base), "r"(wb) : "memory");
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a.visited + (size_t)g * a.gstride + base), "r"(wb)
+               : "memory");
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a.deg + base), "r"(db) : "memory");
 }
 
 template <typename T>
@@ -1421,6 +1434,13 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
       }
       if (a.ctrl[g].done) continue;  // finished before this launch (stable)
       const uint32_t tix = (uint32_t)(w % tpg);
+      if (tid == 0 && !sparse) {
+        // the commit streams S_l, visited and the degrees of its tiles: ask the TMA unit to
+        // prefetch this group's tile two tiles (of this CTA) ahead into L2
+        // (cp.async.bulk.prefetch.L2), so its loads hit L2 instead of waiting on DRAM
+        const size_t tn = (size_t)tix + 2 * (size_t)gridDim.x;
+        if (tn < tpg) prefetch_commit_tile(a, g, lc, tn * CTILE);
+      }
       commit_tile(a, cm, g, lc, (size_t)tix * CTILE, nf, mf, newp, nacc, tix % SAMPLE_TILES == 0, bc, sparse);
       ++ntiles;
     }

@@ -50,7 +50,7 @@ def parse(argv=None):
     ap.add_argument("--direction", default="auto")
     ap.add_argument("--alpha", type=float, default=4.0)
     ap.add_argument("--beta", type=float, default=24.0)
-    ap.add_argument("--split-div", type=float, default=64.0)
+    ap.add_argument("--split-div", type=float, default=512.0)
     ap.add_argument("--group-bits", type=int, default=0, help="instances per group (0 = the config's, 128)")
     ap.add_argument("--plan-hops", type=int, default=2, help="GroupBy hub radius (1 = the literal steps, 2 = 2-hop anchors, P:L577)")
     ap.add_argument("--max-depth", type=int, default=0, help="k-hop mode (the 3-hop index of §8.7): 0 = plain BFS")
@@ -247,7 +247,11 @@ class Workload:
                            max_depth=(args.max_depth or None))
 
     def step_sources(self, k: int) -> np.ndarray:
-        return self.s_plan[self.sched.step_rows(k)]
+        key = (k * self.sched.groups_per_step) % len(self.sched.share)
+        cache = self.__dict__.setdefault("_src", {})
+        if key not in cache:
+            cache[key] = np.ascontiguousarray(self.s_plan[self.sched.step_rows(k)], dtype=np.uint32)
+        return cache[key]
 
 
 def relaunch(args) -> int:
@@ -324,7 +328,9 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
     ev0.record(stream)
+    wall0 = time.perf_counter()
     sts = [do_step(args.warmup + k, True) for k in range(args.steps)]
+    py_wall_ms = (time.perf_counter() - wall0) * 1e3
     ev1.record(stream)
     torch.cuda.synchronize()
     clocks = sampler.stop()
@@ -420,6 +426,10 @@ def main():
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "timeline": {"timed_ms": round(max_ms, 3), "traverse_ms": round(traverse_ms, 3),
                          "level_gap_ms": round(sum(s.level_gap_ms for s in sts), 3),
+                         "host": {"setup_ms": round(sum(s.host_setup_ms for s in sts), 3),
+                                  "wait_ms": round(sum(s.host_wait_ms for s in sts), 3),
+                                  "in_library_ms": round(sum(s.host_total_ms for s in sts), 3),
+                                  "python_wall_ms": round(py_wall_ms, 3)},
                          "note": "traverse = device windows of the ibfs_run_ex calls; level_gap = device idle "
                                  "between consecutive level kernels (in-kernel globaltimer); the rest of "
                                  "timed_ms is between calls / batches"},

@@ -177,7 +177,7 @@ typedef struct {
      instance) run top-down in the same launch. */
   uint32_t split;             /* IBFS_SPLIT_* (default AUTO) */
   uint32_t split_mod;         /* IBFS_SPLIT_FORCE: instances j with j % split_mod == 0 */
-  float split_div;            /* IBFS_SPLIT_AUTO ratio (default 64) */
+  float split_div;            /* IBFS_SPLIT_AUTO ratio (default 512) */
   /* k-hop mode (the reachability index of §8.7: "computes the first k
      levels BFS for a large amount of selected vertices"; Table 1 uses k = 3).  max_depth
      = k >= 1 stops every group after level k: vertices farther than k hops stay -1 and
@@ -261,6 +261,9 @@ typedef struct {
   uint64_t level_launches_live;  /* level launches in which a group was still running (the
                                     others are look-ahead launches that exit at once) */
   uint64_t words_gathered;       /* sum of ibfs_level_stats.gathered */
+  /* host-side wall clock of the call (diagnostics of the gaps between device work):
+     entry -> the first kernel enqueued, time blocked waiting on the device, entry -> return */
+  double host_setup_ms, host_wait_ms, host_total_ms;
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */
   uint64_t *per_source_digest;  /* [n] sum over reached v of splitmix64((v<<8)|(d+1)) */

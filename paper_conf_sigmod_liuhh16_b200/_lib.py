@@ -64,7 +64,8 @@ class Stats(C.Structure):
                 ("depth_bytes", C.c_uint64), ("level_gap_ms", C.c_double),
                 ("commit_bytes_moved", C.c_uint64), ("depth_rows_bytes", C.c_uint64), ("ms_bytes", C.c_uint64),
                 ("ms_ms", C.c_double), ("ms_launches", C.c_uint64), ("level_launches_live", C.c_uint64),
-                ("words_gathered", C.c_uint64),
+                ("words_gathered", C.c_uint64), ("host_setup_ms", C.c_double), ("host_wait_ms", C.c_double),
+                ("host_total_ms", C.c_double),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),
                 ("level_cap", C.c_uint32), ("per_level", C.c_void_p)]
 

@@ -18,7 +18,9 @@
 #include <cub/device/device_segmented_sort.cuh>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
+#include <exception>
 #include <cstdio>
 #include <cstring>
 #include <cstdlib>
@@ -76,11 +78,12 @@ int guarded(F &&f) {
 struct DeviceScope {
   int prev = -1;
   explicit DeviceScope(int dev) {
-    int n = 0;
-    if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
-      cudaGetLastError();
-      fail(IBFS_E_CUDA, "no CUDA device available (libibfs has no CPU fallback)");
-    }
+    static const int n = [] {
+      int c = 0;
+      if (cudaGetDeviceCount(&c) != cudaSuccess) { cudaGetLastError(); c = 0; }
+      return c;
+    }();
+    if (n == 0) fail(IBFS_E_CUDA, "no CUDA device available (libibfs has no CPU fallback)");
     if (dev < 0 || dev >= n) fail(IBFS_E_INVALID, "device index out of range");
     CK(cudaGetDevice(&prev));
     CK(cudaSetDevice(dev));
@@ -104,12 +107,36 @@ Allocator current_allocator() {
   return g_alloc;
 }
 
-// Device scratch owned by one call: caller allocator if installed, else the stream-
-// ordered pool (cudaMallocAsync; the pool keeps memory across calls).
+// Scratch buffers kept by a graph between calls (the same call shape asks for the same
+// buffers in the same order): a call that finds the cache free takes it for its whole
+// duration and reuses buffer i for its i-th request when it is large enough; a concurrent
+// call on the same graph finds it taken and allocates its own.  Saves the per-call
+// allocate / free round trips (tens of them) between back-to-back calls.
+struct ScratchCache {
+  std::mutex mu;
+  std::vector<std::pair<void *, size_t>> bufs;
+  ~ScratchCache() {
+    for (auto &b : bufs) cudaFree(b.first);
+  }
+};
+
+// Device scratch owned by one call: caller allocator if installed, else the graph's cache
+// when free, else the stream-ordered pool (cudaMallocAsync; the pool keeps memory across
+// calls).
 class Scratch {
  public:
-  Scratch(int dev, cudaStream_t s) : dev_(dev), stream_(s), al_(current_allocator()) {}
+  Scratch(int dev, cudaStream_t s, ScratchCache *cache = nullptr)
+      : dev_(dev), stream_(s), al_(current_allocator()) {
+    if (cache && !al_.alloc && cache->mu.try_lock()) cache_ = cache;
+  }
   ~Scratch() {
+    if (cache_) {
+      // an exception left work in flight on the cached buffers: finish it before the next
+      // call may reuse them
+      if (std::uncaught_exceptions() > 0) cudaStreamSynchronize(stream_);
+      cache_->mu.unlock();
+      return;
+    }
     for (void *p : ptrs_) {
       if (al_.alloc) al_.release(p, dev_, al_.ctx);
       else cudaFreeAsync(p, stream_);
@@ -119,6 +146,23 @@ class Scratch {
   T *get(size_t count) {
     size_t bytes = std::max<size_t>(count * sizeof(T), 256);
     void *p = nullptr;
+    if (cache_) {
+      const size_t i = next_++;
+      if (i < cache_->bufs.size() && cache_->bufs[i].second >= bytes) return static_cast<T *>(cache_->bufs[i].first);
+      if (i < cache_->bufs.size()) {  // too small: replace (the previous call has completed)
+        cudaFree(cache_->bufs[i].first);
+        cache_->bufs[i] = {nullptr, 0};
+      }
+      bytes = (bytes + (1u << 20) - 1) & ~(size_t)((1u << 20) - 1);  // round up: fewer regrowths
+      cudaError_t e = cudaMalloc(&p, bytes);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(IBFS_E_NOMEM, "cudaMalloc(" + std::to_string(bytes) + " bytes) failed");
+      }
+      if (i < cache_->bufs.size()) cache_->bufs[i] = {p, bytes};
+      else cache_->bufs.push_back({p, bytes});
+      return static_cast<T *>(p);
+    }
     if (al_.alloc) {
       p = al_.alloc(bytes, dev_, al_.ctx);
       if (!p) fail(IBFS_E_NOMEM, "caller allocator returned NULL");
@@ -138,6 +182,8 @@ class Scratch {
   cudaStream_t stream_;
   Allocator al_;
   std::vector<void *> ptrs_;
+  ScratchCache *cache_ = nullptr;
+  size_t next_ = 0;
 };
 
 void set_pool_threshold(int dev) {
@@ -204,6 +250,7 @@ struct ibfs_graph {
   int num_sms = 148;
   size_t total_mem = 0;  // device memory (bytes), queried once at load
   int level_blocks_per_sm[3] = {1, 1, 1};  // co-resident level_kernel CTAs per SM (W = 32, 64, 128)
+  ScratchCache scratch;  // run scratch kept between calls (Scratch)
 };
 
 namespace {
@@ -226,6 +273,11 @@ void graph_release(ibfs_graph *g) {
   cudaFree(g->d_rchunks);
   cudaFree(g->d_rhub_vtx);
   cudaFree(g->d_rhub_chunk0);
+  {
+    std::lock_guard<std::mutex> lk(g->scratch.mu);
+    for (auto &b : g->scratch.bufs) cudaFree(b.first);
+    g->scratch.bufs.clear();
+  }
   if (prev >= 0) cudaSetDevice(prev);
   cudaGetLastError();
   delete g;
@@ -284,6 +336,15 @@ __device__ __forceinline__ uint32_t dev_compact_id(const uint32_t *tbase, const 
   uint32_t c = tbase[v >> 7];
   for (uint32_t k = w & ~3u; k < w; ++k) c += __popc(nzbits[k]);
   return c + __popc(nzbits[w] & ((1u << (v & 31)) - 1u));
+}
+
+// the run's sources in compacted ids (NO_VERTEX for an isolated source)
+__global__ void compact_sources_kernel(const uint32_t *src, uint32_t n, const uint32_t *tbase, const uint32_t *nzbits,
+                                       uint32_t *csrc) {
+  for (uint32_t r = blockIdx.x * blockDim.x + threadIdx.x; r < n; r += gridDim.x * blockDim.x) {
+    const uint32_t v = src[r];
+    csrc[r] = ((nzbits[v >> 5] >> (v & 31)) & 1u) ? dev_compact_id(tbase, nzbits, v) : NO_VERTEX;
+  }
 }
 
 __global__ void compact_rows_kernel(const unsigned long long *off, uint32_t nv, const uint32_t *tbase,
@@ -977,7 +1038,7 @@ extern "C" void ibfs_run_opts_default(ibfs_run_opts *o) {
   o->beta = 24.0f;
   o->split = IBFS_SPLIT_AUTO;
   o->split_mod = 2;
-  o->split_div = 64.0f;
+  o->split_div = 512.0f;  // A/B sweep, profiles/r02/split_div.md
 }
 
 namespace {
@@ -1084,9 +1145,20 @@ struct EventTimer {
   }
 };
 
+using HostClock = std::chrono::steady_clock;
+double ms_since(HostClock::time_point t0) {
+  return std::chrono::duration<double, std::milli>(HostClock::now() - t0).count();
+}
+// blocks on an event, adding the blocked time to *wait_ms
+void wait_event(cudaEvent_t e, double *wait_ms) {
+  const auto t = HostClock::now();
+  CK(cudaEventSynchronize(e));
+  *wait_ms += ms_since(t);
+}
+
 template <typename T>
-void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *csources, uint32_t n,
-               int8_t *out_depths, const ibfs_run_opts &o, ibfs_stats *stats) {
+void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
+               int8_t *out_depths, const ibfs_run_opts &o, ibfs_stats *stats, HostClock::time_point t_entry) {
   constexpr int W = WordBits<T>::value;
   constexpr size_t B = sizeof(T);
   cudaStream_t stream = (cudaStream_t)o.cuda_stream;
@@ -1120,11 +1192,12 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   uint32_t R = 4;
   while (R < 24 && need(G, R + 1) <= budget) ++R;  // > R-2 levels: flushed ring rounds
 
-  Scratch sc(g->device, stream);
+  Scratch sc(g->device, stream, const_cast<ScratchCache *>(&g->scratch));
   uint32_t *d_src = sc.get<uint32_t>(n);
   CK(cudaMemcpyAsync(d_src, sources, (size_t)n * 4, cudaMemcpyDefault, stream));
   uint32_t *d_csrc = sc.get<uint32_t>(n);
-  CK(cudaMemcpyAsync(d_csrc, csources, (size_t)n * 4, cudaMemcpyDefault, stream));
+  compact_sources_kernel<<<(n + 255) / 256, 256, 0, stream>>>(d_src, n, g->d_tbase, g->d_nzbits, d_csrc);
+  CK(cudaGetLastError());
   T *visited = sc.get<T>(G * gstride);
   T *ring = sc.get<T>((size_t)R * G * gstride);
   uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
@@ -1251,8 +1324,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     cudaEvent_t done = nullptr;
   } pend;
   // host side of a finished batch: per-source outputs, level records, byte models, times
+  double wait_ms = 0, setup_ms = -1;
   auto harvest = [&](const Pending &pb) {
-    CK(cudaEventSynchronize(pb.done));
+    wait_event(pb.done, &wait_ms);
     const Slot &sl = slots[pb.slot];
     const uint32_t gb0 = pb.gb0, Gb = pb.Gb, rows_in_batch = pb.rows;
     const int level = pb.level;
@@ -1346,6 +1420,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
       cudaEvent_t i0 = nullptr, i1 = nullptr;
       if (o.timing) { i0 = timer.next(); i1 = timer.next(); CK(cudaEventRecord(i0, stream)); }
       uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nva + BLOCK - 1) / BLOCK, std::max<uint32_t>(1, 2048 / Gb)));
+      if (setup_ms < 0) setup_ms = ms_since(t_entry);
       init_ctrl_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
       init_state_kernel<T><<<dim3(bx, Gb), BLOCK, 0, stream>>>(a, first_dir);
       init_sources_kernel<T><<<Gb, 128, 0, stream>>>(a, first_dir);
@@ -1358,7 +1433,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
     bool batch_iso = false;  // a source of this batch is isolated (its own zero is a fix-up)
-    for (uint32_t r = 0; r < rows_in_batch; ++r) batch_iso |= csources[(size_t)gb0 * W + r] == NO_VERTEX;
+    for (uint32_t r = 0; r < rows_in_batch; ++r) {
+      const uint32_t v = sources[(size_t)gb0 * W + r];
+      batch_iso |= ((g->h_nzbits[v >> 5] >> (v & 31)) & 1u) == 0;
+    }
     auto flush = [&](int l1, bool final_flush) {
       cudaEvent_t d0 = nullptr, d1 = nullptr, m0 = nullptr, m1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
@@ -1430,7 +1508,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
       ++chunk;
       level = lend;
       if (chunk >= 2) {
-        CK(cudaEventSynchronize(chk_ev[chunk - 2]));
+        wait_event(chk_ev[chunk - 2], &wait_ms);
         if (h_done[chunk - 2] >= Gb) break;
       }
     }
@@ -1494,6 +1572,9 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
   st.n_groups = n_groups;
   st.n_launches = launches;
   st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes + st.depth_bytes + st.ms_bytes;
+  st.host_setup_ms = setup_ms;
+  st.host_wait_ms = wait_ms;
+  st.host_total_ms = ms_since(t_entry);
   if (stats) {
     st.per_source_m = stats->per_source_m;
     st.per_source_digest = stats->per_source_digest;
@@ -1664,6 +1745,7 @@ void run_joint(const ibfs_graph *g, const uint32_t *sources, const uint32_t *cso
 
 extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_t n, uint32_t group_bits,
                            int8_t *out_depths, const ibfs_run_opts *opts, ibfs_stats *stats) {
+  const auto t_entry = HostClock::now();
   return guarded([&] {
     if (!g) fail(IBFS_E_INVALID, "graph is NULL");
     if (group_bits != 32 && group_bits != 64 && group_bits != 128) fail(IBFS_E_INVALID, "group_bits must be 32, 64 or 128");
@@ -1698,15 +1780,20 @@ extern "C" int ibfs_run_ex(const ibfs_graph *g, const uint32_t *sources, uint32_
     // stream (ordered after the work that wrote them; torch streams are non-blocking
     // with respect to the legacy default stream)
     std::vector<uint32_t> hs(n), hcs(n);
-    CK(cudaMemcpyAsync(hs.data(), sources, (size_t)n * 4, cudaMemcpyDefault, (cudaStream_t)o.cuda_stream));
-    CK(cudaStreamSynchronize((cudaStream_t)o.cuda_stream));
+    if (is_device_ptr(sources)) {
+      CK(cudaMemcpyAsync(hs.data(), sources, (size_t)n * 4, cudaMemcpyDeviceToHost, (cudaStream_t)o.cuda_stream));
+      CK(cudaStreamSynchronize((cudaStream_t)o.cuda_stream));
+    } else {
+      std::memcpy(hs.data(), sources, (size_t)n * 4);
+    }
     for (uint32_t r = 0; r < n; ++r)
       if (hs[r] >= g->nv) fail(IBFS_E_INVALID, "source id >= nv");
-    for (uint32_t r = 0; r < n; ++r) hcs[r] = host_compact_id(g, hs[r]);
-    if (o.engine == IBFS_ENGINE_JOINT) run_joint(g, hs.data(), hcs.data(), n, group_bits, out_depths, o, stats);
-    else if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
-    else if (group_bits == 64) run_typed<unsigned long long>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
-    else run_typed<u128>(g, hs.data(), hcs.data(), n, out_depths, o, stats);
+    if (o.engine == IBFS_ENGINE_JOINT) {
+      for (uint32_t r = 0; r < n; ++r) hcs[r] = host_compact_id(g, hs[r]);
+      run_joint(g, hs.data(), hcs.data(), n, group_bits, out_depths, o, stats);
+    } else if (group_bits == 32) run_typed<uint32_t>(g, hs.data(), n, out_depths, o, stats, t_entry);
+    else if (group_bits == 64) run_typed<unsigned long long>(g, hs.data(), n, out_depths, o, stats, t_entry);
+    else run_typed<u128>(g, hs.data(), n, out_depths, o, stats, t_entry);
   });
 }
 

@@ -105,8 +105,13 @@ class GroupSchedule:
         return np.asarray([self.share[(k * G + i) % m] for i in range(G)], dtype=np.int64)
 
     def step_rows(self, k: int) -> np.ndarray:
-        """Indices into the plan-ordered source list of step k, in run order."""
-        return rows_of_groups(self.step_groups(k), self.n, self.group_bits)
+        """Indices into the plan-ordered source list of step k, in run order (steps repeat
+        with period len(share)/gcd: memoised)."""
+        key = (k * self.groups_per_step) % len(self.share)
+        cache = self.__dict__.setdefault("_rows", {})
+        if key not in cache:
+            cache[key] = rows_of_groups(self.step_groups(k), self.n, self.group_bits)
+        return cache[key]
 
 
 def gather_results(n: int, rows: np.ndarray, m_local, dig_local, ms: float, world: int = 1,

@@ -16,6 +16,8 @@ import numpy as np
 from . import _lib
 from ._lib import check
 
+_STAT_FIELDS = tuple(f for f, _ in _lib.Stats._fields_
+                     if f not in ("per_source_m", "per_source_digest", "level_cap", "per_level"))
 _DIRS = {"auto": _lib.DIR_AUTO, "td": _lib.DIR_TD_ONLY, "bu_from": _lib.DIR_BU_FROM,
          "schedule": _lib.DIR_SCHEDULE}
 _PLAN_MODES = {"groupby": 0, "random": 1, "identity": 2}
@@ -96,6 +98,9 @@ class RunStats:
     ms_launches: int
     level_launches_live: int
     words_gathered: int
+    host_setup_ms: float
+    host_wait_ms: float
+    host_total_ms: float
     per_source_m: np.ndarray | None = None
     per_source_digest: np.ndarray | None = None
     per_level: list = field(default_factory=list)
@@ -214,7 +219,7 @@ class Graph:
             schedule: str | None = None, bu_from: int = 2, alpha: float = 4.0, beta: float = 24.0,
             groups_in_flight: int = 0, stream=None, timing: bool = False, want_m: bool = True,
             want_digest: bool = False, level_cap: int = 130, split: str = "auto",
-            split_mod: int = 2, split_div: float = 64.0, max_depth: int | None = None,
+            split_mod: int = 2, split_div: float = 512.0, max_depth: int | None = None,
             engine: str = "bitwise", late_cap: int = 0):
         """n concurrent BFS instances; returns (depths, RunStats).
 
@@ -284,8 +289,7 @@ class Graph:
         st.per_level = C.cast(lv, C.c_void_p)
         check(lib.ibfs_run_ex(self._h, ps if n else None, n, int(group_bits), po, C.byref(opts),
                               C.byref(st)))
-        rs = RunStats(**{f: getattr(st, f) for f, _ in _lib.Stats._fields_
-                         if f not in ("per_source_m", "per_source_digest", "level_cap", "per_level")})
+        rs = RunStats(**{f: getattr(st, f) for f in _STAT_FIELDS})
         rs.per_source_m = m_arr[:n] if want_m else None
         rs.per_source_digest = d_arr[:n] if want_digest else None
         rs.per_level = [

@@ -33,10 +33,11 @@ import ibfs_gen  # noqa: E402
 import oracle  # noqa: E402
 
 GOLDEN = os.path.join(ROOT, "tests", "golden")
-CKPT = os.path.join(ROOT, "gpurun_out", "golden_ckpt")
+CKPT = os.path.join(ROOT, "gpurun_out", "golden_ckpt")  # --ckpt overrides
 
 
-def make(name: str, threads: int, chunk: int) -> str:
+def make(name: str, threads: int, chunk: int, reverse: bool = False, extra_ckpt=(),
+         assemble_only: bool = False) -> str:
     cfg = ibfs_gen.CONFIGS[name]
     t0 = time.time()
     el = cfg.edges(threads=threads)
@@ -52,14 +53,27 @@ def make(name: str, threads: int, chunk: int) -> str:
     ecc = np.zeros(n, dtype=np.int32)
     reached = np.zeros(n, dtype=np.uint64)
     os.makedirs(CKPT, exist_ok=True)
-    for lo in range(0, n, chunk):
+    starts = list(range(0, n, chunk))
+    if reverse:
+        starts = starts[::-1]
+    missing = 0
+    for lo in starts:
         hi = min(n, lo + chunk)
+        got = False
+        for d in [CKPT] + list(extra_ckpt):
+            ck = os.path.join(d, f"{name}_{lo}_{hi}.npz")
+            if os.path.exists(ck):
+                z = np.load(ck)
+                if np.array_equal(z["sources"], src[lo:hi]):
+                    m_s[lo:hi], dig[lo:hi], ecc[lo:hi], reached[lo:hi] = z["m_s"], z["digest"], z["ecc"], z["reached"]
+                    got = True
+                    break
+        if got:
+            continue
+        if assemble_only:
+            missing += 1
+            continue
         ck = os.path.join(CKPT, f"{name}_{lo}_{hi}.npz")
-        if os.path.exists(ck):
-            z = np.load(ck)
-            if np.array_equal(z["sources"], src[lo:hi]):
-                m_s[lo:hi], dig[lo:hi], ecc[lo:hi], reached[lo:hi] = z["m_s"], z["digest"], z["ecc"], z["reached"]
-                continue
         t1 = time.time()
         r = og.bfs(src[lo:hi], want_depths=False, threads=threads)
         if r.status != 0:
@@ -69,6 +83,9 @@ def make(name: str, threads: int, chunk: int) -> str:
         dt = time.time() - t1
         print(f"[{name}] sources [{lo}, {hi}) in {dt:.1f}s  ({float(r.m_s.sum()) / dt / 1e9:.3f} GTEPS)",
               flush=True)
+    if missing:
+        print(f"[{name}] {missing} chunks missing: no golden written", flush=True)
+        return ""
     out = os.path.join(GOLDEN, f"{name}_ms_digest.npz")
     np.savez_compressed(
         out, sources=src, m_s=m_s, digest=dig, ecc=ecc, reached=reached,
@@ -84,10 +101,17 @@ def main():
     ap.add_argument("configs", nargs="+")
     ap.add_argument("--threads", type=int, default=os.cpu_count() or 1)
     ap.add_argument("--chunk", type=int, default=0, help="sources per checkpoint (0 = per config)")
+    ap.add_argument("--ckpt", default=None, help="checkpoint directory (default gpurun_out/golden_ckpt)")
+    ap.add_argument("--extra-ckpt", action="append", default=[], help="more checkpoint directories to read")
+    ap.add_argument("--reverse", action="store_true", help="compute the chunks from the last one down")
+    ap.add_argument("--assemble", action="store_true", help="only assemble existing chunks")
     a = ap.parse_args()
+    if a.ckpt:
+        global CKPT
+        CKPT = os.path.abspath(a.ckpt)
     for name in a.configs:
         chunk = a.chunk or {"c5": 64, "c3": 128, "c4": 16384}.get(name, 1 << 30)
-        make(name, a.threads, chunk)
+        make(name, a.threads, chunk, a.reverse, a.extra_ckpt, a.assemble)
 
 
 if __name__ == "__main__":

@@ -184,6 +184,7 @@ def make_roofline(config, sts, step_ms):
         "level": (S("expand_bytes") + S("commit_bytes"), S("level_ms"), S("level_launches_live"), S("level_launches")),
         "depth": (S("depth_bytes"), S("depth_ms"), S("depth_launches"), S("depth_launches")),
         "ms": (S("ms_bytes"), S("ms_ms"), S("ms_launches"), S("ms_launches")),
+        "clean": (S("clean_bytes"), S("clean_ms"), S("clean_launches"), S("clean_launches")),
     }
     dom = max(kern, key=lambda k: kern[k][1])
     b, ms, live, nl = kern[dom]
@@ -199,7 +200,9 @@ def make_roofline(config, sts, step_ms):
           "algorithmic_bytes_per_launch": (b / live if live else None),
           "launches": nl, "launches_live": live,
           "model": "DESIGN.md §5 = SURVEY.md §8(d): expand 8+B per frontier, 4+B per inspection, B per write; "
-                   "commit 3B per vertex (dense scan) + B per new vertex; depth rows i*|V| + B per loaded snapshot",
+                   "commit 2B per vertex (dense scan; the clean ring clears each read slot once, in the clean "
+                   "kernel: B per vertex and loaded level) + B per new vertex; depth rows i*|V| + B per "
+                   "loaded snapshot",
           "share_of_step": round(ms / step_ms, 4) if step_ms else None,
           "all_kernels": {k: {"GB/s": gbs(v[0], v[1]), "ms": round(v[1], 3), "launches": v[3], "live": v[2],
                               "bytes_per_live_launch": (v[0] / v[2] if v[2] else None)} for k, v in kern.items()},

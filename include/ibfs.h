@@ -245,15 +245,17 @@ typedef struct {
                    (adjacency entry); per gathered neighbour word B (a bottom-up neighbour
                    is read only when the frontier bitmap holds it); per S_l write B; a
                    bottom-up level reads the frontier bitmap (nva/8) once;
-     commit_bytes  the §8(d) dense-scan model: 3B per vertex and level (S_l and visited
-                   read, the next slot cleared) + B per vertex with new bits + the frontier
-                   bitmap written (nva/8);
+     commit_bytes  the §8(d) dense-scan model: 2B per vertex and level (S_l and visited
+                   read; 3B with IBFS_CLEAN_RING=0, where the commit also clears the next
+                   slot) + B per vertex with new bits + the frontier bitmap written (nva/8);
      commit_bytes_moved  what the commits actually stream: a sparse commit
                    reads the chunk map, the marked chunks (bounded by the level's writes)
                    and clears the next slot;
      depth_bytes   depth_kernel only: int8 rows written (depth_rows_bytes) + B per vertex,
                    group and loaded snapshot level (levels 1..last_level of each group,
-                   skipped levels excluded) + the late-list fix-ups;
+                   skipped levels excluded) + the late-list fix-ups; with the clean ring
+                   at W = 128 the depth kernel also zeroes each loaded run (B per vertex,
+                   group and loaded level, bulk stores) and clean_bytes excludes them;
      ms_bytes      the m_s pass: (B + 4) per vertex and group (final words + degrees). */
   uint64_t commit_bytes_moved, depth_rows_bytes, ms_bytes;
   double ms_ms;                  /* m_s pass + late-list / isolated-source fix-ups (opts.timing) */
@@ -264,6 +266,11 @@ typedef struct {
   /* host-side wall clock of the call (diagnostics of the gaps between device work):
      entry -> the first kernel enqueued, time blocked waiting on the device, entry -> return */
   double host_setup_ms, host_wait_ms, host_total_ms;
+  /* clean ring: ring_clean_kernel zeroes the snapshot slots the depth pass
+     read (B per vertex, group and loaded level) and late_fix_kernel the skipped levels'
+     entries (B each), so no commit clears a slot; clean_ms is CUDA-event time (opts.timing) */
+  double clean_ms;
+  uint64_t clean_launches, clean_bytes;
   /* optional caller-provided HOST arrays (NULL = not wanted) */
   uint64_t *per_source_m;       /* [n] m_s */
   uint64_t *per_source_digest;  /* [n] sum over reached v of splitmix64((v<<8)|(d+1)) */

@@ -66,6 +66,7 @@ class Stats(C.Structure):
                 ("ms_ms", C.c_double), ("ms_launches", C.c_uint64), ("level_launches_live", C.c_uint64),
                 ("words_gathered", C.c_uint64), ("host_setup_ms", C.c_double), ("host_wait_ms", C.c_double),
                 ("host_total_ms", C.c_double),
+                ("clean_ms", C.c_double), ("clean_launches", C.c_uint64), ("clean_bytes", C.c_uint64),
                 ("per_source_m", C.c_void_p), ("per_source_digest", C.c_void_p),
                 ("level_cap", C.c_uint32), ("per_level", C.c_void_p)]
 

@@ -115,6 +115,7 @@ Allocator current_allocator() {
 struct ScratchCache {
   std::mutex mu;
   std::vector<std::pair<void *, size_t>> bufs;
+  std::vector<char> zero;  // buffer i is known to be all zero (the clean ring)
   ~ScratchCache() {
     for (auto &b : bufs) cudaFree(b.first);
   }
@@ -142,12 +143,34 @@ class Scratch {
       else cudaFreeAsync(p, stream_);
     }
   }
+  // A buffer that must be all zero: from the cache when the previous call left it zero
+  // (mark_zero), else cleared here on the stream.  Returns its cache index (or -1).
+  template <typename T>
+  T *get_zeroed(size_t count, int *idx) {
+    const size_t i = next_;
+    const bool was_zero = cache_ && i < cache_->zero.size() && cache_->zero[i] && i < cache_->bufs.size() &&
+                          cache_->bufs[i].second >= std::max<size_t>(count * sizeof(T), 256);
+    T *p = get<T>(count);  // clears the flag
+    // the whole allocation (a cached buffer may be larger than this request; a later call
+    // may use more of it while the flag says zero)
+    const size_t whole = cache_ ? cache_->bufs[i].second : std::max<size_t>(count * sizeof(T), 256);
+    if (!was_zero) CK(cudaMemsetAsync(p, 0, whole, stream_));
+    *idx = cache_ ? (int)i : -1;
+    return p;
+  }
+  // the call leaves buffer idx all zero again (only after its work completed normally)
+  void mark_zero(int idx) {
+    if (!cache_ || idx < 0) return;
+    if (cache_->zero.size() <= (size_t)idx) cache_->zero.resize(idx + 1, 0);
+    cache_->zero[idx] = 1;
+  }
   template <typename T>
   T *get(size_t count) {
     size_t bytes = std::max<size_t>(count * sizeof(T), 256);
     void *p = nullptr;
     if (cache_) {
       const size_t i = next_++;
+      if (i < cache_->zero.size()) cache_->zero[i] = 0;  // handed out: contents unknown from now
       if (i < cache_->bufs.size() && cache_->bufs[i].second >= bytes) return static_cast<T *>(cache_->bufs[i].first);
       if (i < cache_->bufs.size()) {  // too small: replace (the previous call has completed)
         cudaFree(cache_->bufs[i].first);
@@ -250,6 +273,8 @@ struct ibfs_graph {
   int num_sms = 148;
   size_t total_mem = 0;  // device memory (bytes), queried once at load
   int level_blocks_per_sm[3] = {1, 1, 1};  // co-resident level_kernel CTAs per SM (W = 32, 64, 128)
+  int dtma_blocks_per_sm[3] = {1, 1, 1};   // depth_tma_kernel (grid = SMs x this / groups)
+  int depth_blocks_per_sm[3] = {1, 1, 1};  // depth_kernel
   ScratchCache scratch;  // run scratch kept between calls (Scratch)
 };
 
@@ -532,6 +557,31 @@ void finish_graph(ibfs_graph *g) {
   g->level_blocks_per_sm[1] = std::max(1, occ);
   CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, level_kernel<u128>, BLOCK, sizeof(TileQueue<u128>)));
   g->level_blocks_per_sm[2] = std::max(1, occ);
+  // the depth kernels are persistent over their tiles: their grids are sized from the
+  // occupancy the shared-memory footprint really allows (not from the launch bounds)
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, depth_tma_kernel<uint32_t>, DTHREADS + 32,
+                                                   depth_tma_smem_bytes<uint32_t>()));
+  g->dtma_blocks_per_sm[0] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, depth_tma_kernel<unsigned long long>, DTHREADS + 32,
+                                                   depth_tma_smem_bytes<unsigned long long>()));
+  g->dtma_blocks_per_sm[1] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, depth_tma_kernel<u128>, DTHREADS + 32,
+                                                   depth_tma_smem_bytes<u128>()));
+  g->dtma_blocks_per_sm[2] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, depth_kernel<uint32_t>, DTHREADS + 32,
+                                                   depth_smem_bytes<uint32_t>()));
+  g->depth_blocks_per_sm[0] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, depth_kernel<unsigned long long>, DTHREADS + 32,
+                                                   depth_smem_bytes<unsigned long long>()));
+  g->depth_blocks_per_sm[1] = std::max(1, occ);
+  CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, depth_kernel<u128>, DTHREADS + 32, depth_smem_bytes<u128>()));
+  g->depth_blocks_per_sm[2] = std::max(1, occ);
+  if (std::getenv("IBFS_VERBOSE"))
+    std::fprintf(stderr, "ibfs: CTAs/SM level %d/%d/%d depth_tma %d/%d/%d depth %d/%d/%d (W=32/64/128); smem depth_tma %zu B\n",
+                 g->level_blocks_per_sm[0], g->level_blocks_per_sm[1], g->level_blocks_per_sm[2],
+                 g->dtma_blocks_per_sm[0], g->dtma_blocks_per_sm[1], g->dtma_blocks_per_sm[2],
+                 g->depth_blocks_per_sm[0], g->depth_blocks_per_sm[1], g->depth_blocks_per_sm[2],
+                 depth_tma_smem_bytes<u128>());
   set_pool_threshold(dev);
 }
 
@@ -1072,6 +1122,40 @@ uint32_t bu_probe_mode() {
   return m;
 }
 
+// Clean ring unless IBFS_CLEAN_RING=0 (A/B runs: the commits clear the next
+// slot every level, as in round 1).  IBFS_CHECK_RING=1 (tests) verifies after every call
+// that the ring is all zero again and fails with IBFS_E_CUDA otherwise.
+bool clean_ring_enabled() {
+  static const bool on = [] {
+    const char *e = std::getenv("IBFS_CLEAN_RING");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+// IBFS_FUSED_CLEAN=0 (A/B runs): zero the read slots in ring_clean_kernel even where the
+// depth kernel could do it with bulk stores.
+bool fused_clean_enabled() {
+  static const bool on = [] {
+    const char *e = std::getenv("IBFS_FUSED_CLEAN");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+bool check_ring_enabled() {
+  const char *e = std::getenv("IBFS_CHECK_RING");
+  return e && e[0] == '1';
+}
+
+// IBFS_SPLIT_REL=x (A/B runs): in a split bottom-up level, also expand top-down every
+// instance whose sampled frontier edge count is below 1/x of the group's largest (0 = off).
+float split_rel_default() {
+  static const float v = [] {
+    const char *e = std::getenv("IBFS_SPLIT_REL");
+    return e ? (float)std::atof(e) : 0.f;
+  }();
+  return v;
+}
+
 bool depth_tma_enabled() {
   static const bool on = [] {
     const char *e = std::getenv("IBFS_DEPTH_TMA");
@@ -1199,7 +1283,11 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   compact_sources_kernel<<<(n + 255) / 256, 256, 0, stream>>>(d_src, n, g->d_tbase, g->d_nzbits, d_csrc);
   CK(cudaGetLastError());
   T *visited = sc.get<T>(G * gstride);
-  T *ring = sc.get<T>((size_t)R * G * gstride);
+  // clean ring: all slots zero at batch start, zeroed again after the depth
+  // rows are written; a ring the previous call did not leave zero is cleared once here
+  const bool clean_ring = clean_ring_enabled();
+  int ring_idx = -1;
+  T *ring = clean_ring ? sc.get_zeroed<T>((size_t)R * G * gstride, &ring_idx) : sc.get<T>((size_t)R * G * gstride);
   uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   uint32_t *buq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
   const uint32_t nchunk32 = (nva + 31) / 32;
@@ -1291,6 +1379,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   a.late = late;
   a.late_n = late_n;
   a.late_cap = late_cap;
+  a.clean_ring = clean_ring ? 1u : 0u;
   a.n_iso = nv - nva;
   a.pol.mode = o.direction;
   a.pol.bu_from = o.bu_from;
@@ -1303,6 +1392,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   a.pol.split_div = o.split_div;
   a.pol.max_depth = o.max_depth;
   a.pol.bu_probe = bu_probe_mode();
+  a.pol.split_rel = split_rel_default();
   a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
   for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
   uint32_t first_dir = 0;
@@ -1311,7 +1401,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
 
   const int level_grid = g->num_sms * g->level_blocks_per_sm[W == 32 ? 0 : (W == 64 ? 1 : 2)];
   EventTimer timer(dc, true), chk(dc, false);
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin, kms, kcopy;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> win, klev, kinit, kdep, kfin, kms, kcopy, kcl;
   ibfs_stats st{};
   uint64_t launches = 0;
   bool range_error = false;
@@ -1321,6 +1411,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
     bool valid = false;
     uint32_t gb0 = 0, Gb = 0, rows = 0;
     int level = 0, slot = 0;
+    int fused_from = 1 << 30;  // levels >= this were zeroed by the depth kernel (fused clean)
     cudaEvent_t done = nullptr;
   } pend;
   // host side of a finished batch: per-source outputs, level records, byte models, times
@@ -1362,7 +1453,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
         // commit (§8(d) dense scan): S_l and visited read, the next slot cleared, visited
         // written where new, the frontier bitmap written (nva / 8 B).
         uint64_t eb = (8 + B) * L.proc + 4 * L.insp + B * L.gath + B * L.writes + (L.dir == 2 ? (uint64_t)nchunk32 * 4 : 0);
-        uint64_t cb = (uint64_t)nva * (3 * B) + B * L.nf + (uint64_t)nchunk32 * 4;
+        uint64_t cb = (uint64_t)nva * ((clean_ring ? 2 : 3) * B) + B * L.nf + (uint64_t)nchunk32 * 4;
         st.expand_bytes += eb;
         st.commit_bytes += cb;
         // what the commit streams: dense -- S_l, visited, the cleared slot, degrees (and
@@ -1371,9 +1462,16 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
         const uint64_t degb = g->directed ? 8 : 4;
         if (L.flags & 2u) {
           const uint64_t chunks = std::min<uint64_t>(L.writes, nchunk32);
-          st.commit_bytes_moved += nchunk32 * 5ull + chunks * 32 * (2 * B + degb) + (uint64_t)nva * B + B * L.nf;
+          st.commit_bytes_moved += nchunk32 * 5ull + chunks * 32 * (2 * B + degb) + (clean_ring ? 0 : (uint64_t)nva * B) + B * L.nf;
         } else {
-          st.commit_bytes_moved += (uint64_t)nva * (3 * B + degb) + nchunk32 * 5ull + B * L.nf;
+          st.commit_bytes_moved += (uint64_t)nva * ((clean_ring ? 2 : 3) * B + degb) + nchunk32 * 5ull + B * L.nf;
+        }
+        // clean ring: a loaded level's slot is zeroed after the depth pass (B per vertex);
+        // a skipped level's late entries are zeroed by the fix-up (B per entry)
+        if (clean_ring) {
+          if (L.flags & 1u) st.clean_bytes += (uint64_t)L.nf * B;
+          else if (l >= pb.fused_from) st.depth_bytes += (uint64_t)nva * B;  // the depth kernel's zero stores
+          else st.clean_bytes += (uint64_t)nva * B;
         }
         // depth kernel: a loaded level's snapshot is read once; a skipped level's new
         // vertices (<= nf) are read back from the late list (entry + word) instead
@@ -1427,11 +1525,12 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
       CK(cudaGetLastError());
       launches += 3;
       st.init_launches += 3;
-      st.init_bytes += (uint64_t)Gb * (3 * (uint64_t)nva * B);
+      st.init_bytes += (uint64_t)Gb * ((clean_ring ? 1 : 3) * (uint64_t)nva * B);
       if (o.timing) { CK(cudaEventRecord(i1, stream)); kinit.push_back({i0, i1}); }
     }
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
+    int fused_from = 1 << 30;
     bool batch_iso = false;  // a source of this batch is isolated (its own zero is a fix-up)
     for (uint32_t r = 0; r < rows_in_batch; ++r) {
       const uint32_t v = sources[(size_t)gb0 * W + r];
@@ -1441,13 +1540,16 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
       cudaEvent_t d0 = nullptr, d1 = nullptr, m0 = nullptr, m1 = nullptr;
       if (o.timing) { d0 = timer.next(); d1 = timer.next(); CK(cudaEventRecord(d0, stream)); }
       const uint32_t bx = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
-                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DEPTH_MINB / Gb)));
+                                                                         std::max<uint64_t>(1, (uint64_t)g->num_sms * g->depth_blocks_per_sm[W == 32 ? 0 : (W == 64 ? 1 : 2)] / Gb)));
       const int first = flushed < 0 ? 1 : 0;
       CUtensorMap tmap;
+      bool fused_clean = false;  // the depth kernel zeroes the runs it loaded (clean ring, W = 128)
       if (first && depth_tma_enabled() && make_rows_tensor_map(&tmap, a.out, nv, rows_in_batch, W)) {
+        fused_clean = clean_ring && B == 16 && fused_clean_enabled();
+        if (fused_clean) fused_from = std::min(fused_from, flushed + 1);
         const uint32_t bt = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(((uint64_t)nv + DV - 1) / DV,
-                                                                           std::max<uint64_t>(1, (uint64_t)g->num_sms * IBFS_DTMA_MINB / Gb)));
-        depth_tma_kernel<T><<<dim3(bt, Gb), DTHREADS + 32, depth_tma_smem_bytes<T>(), stream>>>(tmap, a, flushed + 1, l1);
+                                                                           std::max<uint64_t>(1, (uint64_t)g->num_sms * g->dtma_blocks_per_sm[W == 32 ? 0 : (W == 64 ? 1 : 2)] / Gb)));
+        depth_tma_kernel<T><<<dim3(bt, Gb), DTHREADS + 32, depth_tma_smem_bytes<T>(), stream>>>(tmap, a, flushed + 1, l1, fused_clean ? 1 : 0);
       } else {
         depth_kernel<T><<<dim3(bx, Gb), DTHREADS + 32, depth_smem_bytes<T>(), stream>>>(a, flushed + 1, l1, first);
       }
@@ -1474,6 +1576,16 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
         st.ms_bytes += (uint64_t)Gb * nva * (B + 4);
       }
       if (o.timing) { CK(cudaEventRecord(m1, stream)); kms.push_back({m0, m1}); }
+      if (clean_ring && !fused_clean) {  // the read slots back to zero (after late_fix read the skipped entries)
+        cudaEvent_t c0 = nullptr, c1 = nullptr;
+        if (o.timing) { c0 = timer.next(); c1 = timer.next(); CK(cudaEventRecord(c0, stream)); }
+        const uint32_t cx = (uint32_t)std::max<uint64_t>(
+            1, std::min<uint64_t>(((uint64_t)nva * B / 16 + BLOCK) / BLOCK, std::max<uint64_t>(1, (uint64_t)g->num_sms * 8 / Gb)));
+        ring_clean_kernel<T><<<dim3(cx, Gb), BLOCK, 0, stream>>>(a, flushed + 1, l1);
+        launches++;
+        st.clean_launches++;
+        if (o.timing) { CK(cudaEventRecord(c1, stream)); kcl.push_back({c0, c1}); }
+      }
       flushed = l1;
     };
     int level = 1;
@@ -1551,6 +1663,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
     cur.Gb = Gb;
     cur.rows = rows_in_batch;
     cur.level = level;
+    cur.fused_from = fused_from;
     cur.slot = batch_no & 1;
     cur.done = timer.next();  // not from `chk`: its events are recycled every batch
     CK(cudaEventRecord(cur.done, stream));
@@ -1568,10 +1681,22 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   for (auto &p : kdep) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.depth_ms += ms; }
   for (auto &p : kms) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.ms_ms += ms; }
   for (auto &p : kcopy) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.copyout_ms += ms; }
+  for (auto &p : kcl) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.clean_ms += ms; }
+  if (clean_ring && check_ring_enabled()) {
+    CK(cudaMemsetAsync(flags, 0, 4, stream));
+    const size_t n16 = (size_t)R * G * gstride * B / 16;
+    ring_check_kernel<<<(uint32_t)std::min<size_t>((n16 + 255) / 256, 4096), 256, 0, stream>>>(
+        reinterpret_cast<const uint4 *>(ring), n16, flags);
+    uint32_t bad = 0;
+    CK(cudaMemcpyAsync(&bad, flags, 4, cudaMemcpyDeviceToHost, stream));
+    CK(cudaStreamSynchronize(stream));
+    if (bad) fail(IBFS_E_CUDA, "IBFS_CHECK_RING: a ring slot is not zero after the call");
+  }
+  if (clean_ring) sc.mark_zero(ring_idx);  // every batch's clean-up is complete (harvest waited)
   st.depth_bytes += st.depth_rows_bytes;
   st.n_groups = n_groups;
   st.n_launches = launches;
-  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes + st.depth_bytes + st.ms_bytes;
+  st.bytes_algorithmic = st.expand_bytes + st.commit_bytes + st.init_bytes + st.depth_bytes + st.ms_bytes + st.clean_bytes;
   st.host_setup_ms = setup_ms;
   st.host_wait_ms = wait_ms;
   st.host_total_ms = ms_since(t_entry);

@@ -134,6 +134,7 @@ struct Policy {
   float split_div;
   uint32_t max_depth;  // k-hop cap (0 = unbounded)
   uint32_t bu_probe;   // frontier-bitmap probes in BU: 0 never, 1 sparse frontiers (default), 2 always
+  float split_rel;     // > 0: also top-down when m_f(j) * split_rel < max over active j' of m_f(j')
   uint8_t sched[MAXL];  // 0 TD / 1 BU for level l at index l-1
 };
 
@@ -168,6 +169,9 @@ struct BatchArgs {
   unsigned long long *late;  // [gcap][late_cap] (level << 32 | v) new vertices of sparse commits
   uint32_t *late_n;          // [gcap] appended entries (may exceed late_cap: then no more skips)
   uint32_t late_cap;
+  uint32_t clean_ring;  // 1: every ring slot is zero at batch start and is zeroed again after
+                        // its depths are written (ring_clean_kernel, late_fix_kernel), so
+                        // neither init nor the commits clear slots
   uint32_t nchunk32;    // ceil(nva / 32)
   GroupCtrl<T> *ctrl;
   LevelStat *lstat;     // [G][MAXL]
@@ -416,8 +420,10 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
     const bool in = v < a.nva;
     if (in) {
       st(vis + v, z);
-      st(s0 + v, z);
-      st(s1 + v, z);
+      if (!a.clean_ring) {
+        st(s0 + v, z);
+        st(s1 + v, z);
+      }
       if ((v & 31) == 0) {
         a.dirty[(size_t)g * a.nchunk32 + (v >> 5)] = 0;
         a.fbits[(size_t)g * a.nchunk32 + (v >> 5)] = 0u;
@@ -1002,6 +1008,7 @@ struct CommitSmem {
   uint32_t qbase[4];
   float bcnt[WordBits<T>::value];       // sampled per-instance frontier degree sums of this CTA
   uint32_t tdb[WordBits<T>::value / 32];  // split decision (last CTA of a group)
+  uint32_t wmax;                           // max sampled m_f(j) over active j (float bits)
 };
 
 // Per-instance frontier edge counts m_f(j) for the split decision (IBFS_SPLIT_AUTO) are
@@ -1113,7 +1120,7 @@ __device__ __forceinline__ void commit_tile(const BatchArgs<T> &a, CommitSmem<T>
   for (int k = 0; k < CVT; ++k) {
     const size_t v = base + (size_t)k * BLOCK + tid;
     const bool in = v < nv;
-    if (in) st(Z + v, wzero_value<T>());
+    if (in && !a.clean_ring) st(Z + v, wzero_value<T>());
     {  // an unfiltered top-down level may have ORed already-visited bits: mask them
       const T m = wandn(n[k], vv[k]);
       if (in && !weq(m, n[k])) st(N + v, m);
@@ -1285,6 +1292,10 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
   // m_f(j) * split_div exceeds its unexplored edge count m_u(j) = ne - sum of the earlier
   // frontiers' edges (both sampled); FORCE: j % split_mod == 0
   if (tid < W / 32) cm.tdb[tid] = 0;
+  if (tid == 0) cm.wmax = 0u;
+  __syncthreads();
+  if (a.pol.split_rel > 0.f && tid < W && ((wpiece(act, tid >> 5) >> (tid & 31)) & 1u))
+    atomicMax(&cm.wmax, __float_as_uint(*(volatile float *)&c->bitw[tid]));  // w >= 0: bits order as values
   __syncthreads();
   if (tid < W) {
     const float w = *(volatile float *)&c->bitw[tid];
@@ -1296,6 +1307,9 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
     else {
       const double mf = (double)w * SAMPLE, mu = fmax((double)a.pol.ne - (double)cum * SAMPLE, 1.0);
       small = mf * (double)a.pol.split_div < mu;
+      // a laggard among the group's instances keeps every bottom-up scan running to the
+      // end of the row: expand it top-down too (performance only, never the result)
+      if (a.pol.split_rel > 0.f && w * a.pol.split_rel < __uint_as_float(cm.wmax)) small = true;
     }
     if (a.pol.split != 1 && small && ((wpiece(act, tid >> 5) >> (tid & 31)) & 1u))
       atomicOr(&cm.tdb[tid >> 5], 1u << (tid & 31));
@@ -1866,7 +1880,7 @@ __device__ __forceinline__ void sts8(uint32_t a, uint32_t v) {
 // stages (at least one, for its header); only loaded levels occupy slots.
 template <typename T>
 __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DTMA_MINB)
-    depth_tma_kernel(const __grid_constant__ CUtensorMap tmap, BatchArgs<T> a, int l0, int l1) {
+    depth_tma_kernel(const __grid_constant__ CUtensorMap tmap, BatchArgs<T> a, int l0, int l1, int zero_runs) {
   using L = DepthTmaLayout<T>;
   constexpr int W = WordBits<T>::value;
   constexpr int PB = W / 4;   // instances per part
@@ -1875,6 +1889,11 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DTMA_MINB)
   const uint32_t sbase = (smem_u32(dsm_raw) + 127u) & ~127u;
   const uint32_t outb = sbase;  // [2][W][DV] row-major output tiles
   const uint32_t stage_base = sbase + 2 * (uint32_t)L::TILE;
+  // clean ring, fused (W = 128: one 16-byte word per vertex): once the consumers have read
+  // a stage, its snapshot runs have landed in shared memory, so they overwrite the runs in
+  // global memory with zeros (one streaming store per vertex and loaded level, spread over
+  // the consumer threads) and the ring is zero again without a separate pass
+  const bool zr = zero_runs != 0 && sizeof(T) == 16;
   __shared__ __align__(8) unsigned long long s_full[DNS2], s_empty[DNS2];
   __shared__ const T *s_run[DMAXL];  // snapshot array of each loaded level, in level order
   __shared__ uint8_t s_inc[DMAXL];   // its level + 1
@@ -2024,6 +2043,12 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DTMA_MINB)
               }
               reached[r] |= hb;
             }
+          }
+        }
+        if (zr) {  // the stage's runs are in shared memory: zero them in the ring
+          for (uint32_t u = 0; u < nl; ++u) {
+            uint4 *dst = reinterpret_cast<uint4 *>(const_cast<T *>(s_run[b * DLB2 + (int)u]) + hdr.z);
+            for (uint32_t i = (uint32_t)t; i < k; i += DTHREADS) __stcs(dst + i, make_uint4(0u, 0u, 0u, 0u));
           }
         }
         __syncwarp();
@@ -2177,7 +2202,11 @@ __global__ void late_fix_kernel(BatchArgs<T> a, int l0, int l1) {
   const size_t nvv = a.nv;
   if (l0 == 0 && skipped(0) && blockIdx.x == 0)
     for (int j = threadIdx.x; j < rows; j += blockDim.x)
-      if (a.csrc[(size_t)g * W + j] != NO_VERTEX) a.out[((size_t)g * W + j) * nvv + a.src[(size_t)g * W + j]] = 0;
+      if (a.csrc[(size_t)g * W + j] != NO_VERTEX) {
+        a.out[((size_t)g * W + j) * nvv + a.src[(size_t)g * W + j]] = 0;
+        // S_0 holds bits only at the sources (duplicates store the same zero)
+        if (a.clean_ring) st(snap(a, g, 0) + a.csrc[(size_t)g * W + j], wzero_value<T>());
+      }
   const uint32_t n = min(a.late_n[g], a.late_cap);
   const uint32_t ntiles = (uint32_t)((nvv + 127) / 128);
   for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < n; e += gridDim.x * blockDim.x) {
@@ -2185,7 +2214,10 @@ __global__ void late_fix_kernel(BatchArgs<T> a, int l0, int l1) {
     const int l = (int)(ent >> 32);
     const uint32_t v = (uint32_t)ent;
     if (l < l0 || l > last || !skipped(l)) continue;
-    const T x = ldg(snap(a, g, l) + v);
+    // a coherent load: the non-coherent path (ldg) may be scheduled after the clean-ring
+    // store below, which would read the zero
+    T *sp = snap(a, g, l) + v;
+    const T x = ld(sp);
     const size_t col = caller_id(a.tbase, a.nzbits, ntiles, v);
 #pragma unroll
     for (int p = 0; p < W / 32; ++p) {
@@ -2196,7 +2228,43 @@ __global__ void late_fix_kernel(BatchArgs<T> a, int l0, int l1) {
         if (j < rows) a.out[((size_t)g * W + j) * nvv + col] = (int8_t)l;
       }
     }
+    if (a.clean_ring) st(sp, wzero_value<T>());  // the one entry per (level, vertex)
   }
+}
+
+// Clean ring (BatchArgs::clean_ring): after the depth rows of levels [l0, l1] are written,
+// zero the snapshot slots the depth kernel read (every level <= last_level that was not
+// skipped) with 16-byte streaming stores; the skipped levels' few entries were zeroed by
+// late_fix_kernel.  Levels past a group's last_level were never written (the expand of a
+// finished group does not run).  The ring is then all zero again for the next batch, so the
+// commits need not clear the slot of the next level (16 B per vertex and level, sparse
+// tail levels included).
+template <typename T>
+__global__ void __launch_bounds__(BLOCK) ring_clean_kernel(BatchArgs<T> a, int l0, int l1) {
+  const int g = blockIdx.y;
+  if (group_rows(a, g) == 0) return;
+  const GroupCtrl<T> *c = a.ctrl + g;
+  if (c->last_level == 0xffffffffu) return;
+  const int last = min((int)c->last_level, min(l1, 127));
+  const unsigned long long sk0 = c->skip_lv[0], sk1 = c->skip_lv[1];
+  const size_t n16 = (size_t)a.nva * sizeof(T) / 16 + 1;  // slot words rounded up (gstride pads)
+  const size_t stride = (size_t)gridDim.x * BLOCK;
+  const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+  for (int l = l0; l <= last; ++l) {
+    if (((l < 64 ? sk0 >> l : sk1 >> (l - 64)) & 1ull) != 0) continue;
+    uint4 *p = reinterpret_cast<uint4 *>(snap(a, g, l));
+    for (size_t i = (size_t)blockIdx.x * BLOCK + threadIdx.x; i < n16; i += stride) __stcs(p + i, z);
+  }
+}
+
+// IBFS_CHECK_RING (tests): flag = 1 if any of the n16 16-byte words is non-zero.
+__global__ void ring_check_kernel(const uint4 *p, size_t n16, uint32_t *flag) {
+  uint32_t acc = 0;
+  for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += (size_t)gridDim.x * blockDim.x) {
+    const uint4 x = p[i];
+    acc |= x.x | x.y | x.z | x.w;
+  }
+  if (__syncthreads_or(acc != 0) && threadIdx.x == 0) atomicExch(flag, 1u);
 }
 
 __device__ __forceinline__ unsigned long long splitmix64(unsigned long long z) {

@@ -101,6 +101,9 @@ class RunStats:
     host_setup_ms: float
     host_wait_ms: float
     host_total_ms: float
+    clean_ms: float
+    clean_launches: int
+    clean_bytes: int
     per_source_m: np.ndarray | None = None
     per_source_digest: np.ndarray | None = None
     per_level: list = field(default_factory=list)

@@ -6,6 +6,9 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
+# every library call in the tests verifies that it left the snapshot ring all zero (the
+# clean-ring invariant); an unclean slot fails the call
+os.environ.setdefault("IBFS_CHECK_RING", "1")
 
 
 def pytest_configure(config):

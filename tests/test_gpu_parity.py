@@ -320,6 +320,11 @@ def test_depth_above_127_is_range_error():
     with pytest.raises(_lib.IbfsError) as e:
         g.run(np.array([0], dtype=np.uint32), 32)
     assert e.value.code == _lib.IBFS_E_RANGE
+    # the failed call left its ring slots dirty (never marked zero): the next call on the
+    # same graph clears them first (clean ring) and is exact
+    s = np.array([100, 90, 110], dtype=np.uint32)  # max depths 100, 109, 110
+    d, _ = gpu_depths(g, s, 32)
+    np.testing.assert_array_equal(d, oracle.bfs(el, s).depths)
     # a 128-vertex path has max depth 127: fits
     el = ibfs_gen.from_pairs(128, [(i, i + 1) for i in range(127)])
     g = P.Graph.from_edgelist(el)

@@ -12,8 +12,8 @@ fi
 timeout 2400 python -m pytest tests -m gpu -q -x $DESEL > "$OUT/pytest_gpu.log" 2>&1
 echo "rc=$?" >> "$OUT/pytest_gpu.log"
 for c in c5 c4 c3; do
-  for v in "1 1" "1 0" "0 1"; do
-    set -- $v
+  for v in ${VARIANTS:-1_1 1_0 0_1}; do
+    set -- ${v/_/ }
     IBFS_CLEAN_RING=$1 IBFS_FUSED_CLEAN=$2 timeout 900 python bench.py --config $c --no-e2e --no-cpu-baseline --json-out "$OUT/bench_${c}_cr$1_fc$2.json" > "$OUT/bench_${c}_cr$1_fc$2.log" 2>&1
   done
 done

@@ -1132,12 +1132,13 @@ bool clean_ring_enabled() {
   }();
   return on;
 }
-// IBFS_FUSED_CLEAN=0 (A/B runs): zero the read slots in ring_clean_kernel even where the
-// depth kernel could do it with bulk stores.
+// IBFS_FUSED_CLEAN=1 (A/B runs): the depth kernel's consumers zero the runs they read
+// (W = 128) instead of ring_clean_kernel.  Measured (profiles/r02/clean_ring/): c5 depth
+// flush +20.5 ms per 8 steps against 11.5 ms for the separate pass, c3 -1 ms: off by default.
 bool fused_clean_enabled() {
   static const bool on = [] {
     const char *e = std::getenv("IBFS_FUSED_CLEAN");
-    return !(e && e[0] == '0');
+    return e && e[0] == '1';
   }();
   return on;
 }
@@ -1282,10 +1283,13 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   uint32_t *d_csrc = sc.get<uint32_t>(n);
   compact_sources_kernel<<<(n + 255) / 256, 256, 0, stream>>>(d_src, n, g->d_tbase, g->d_nzbits, d_csrc);
   CK(cudaGetLastError());
-  T *visited = sc.get<T>(G * gstride);
+  // clean ring: visited too is all zero between calls (ms_kernel zeroes each word after
+  // reading it), so init only sets the sources
+  const bool clean_ring = clean_ring_enabled();
+  int vis_idx = -1;
+  T *visited = clean_ring ? sc.get_zeroed<T>(G * gstride, &vis_idx) : sc.get<T>(G * gstride);
   // clean ring: all slots zero at batch start, zeroed again after the depth
   // rows are written; a ring the previous call did not leave zero is cleared once here
-  const bool clean_ring = clean_ring_enabled();
   int ring_idx = -1;
   T *ring = clean_ring ? sc.get_zeroed<T>((size_t)R * G * gstride, &ring_idx) : sc.get<T>((size_t)R * G * gstride);
   uint32_t *tdq = sc.get<uint32_t>((size_t)G * std::max<uint32_t>(nva, 1));
@@ -1525,7 +1529,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
       CK(cudaGetLastError());
       launches += 3;
       st.init_launches += 3;
-      st.init_bytes += (uint64_t)Gb * ((clean_ring ? 1 : 3) * (uint64_t)nva * B);
+      st.init_bytes += (uint64_t)Gb * (clean_ring ? (uint64_t)nchunk32 * 5 : 3 * (uint64_t)nva * B);
       if (o.timing) { CK(cudaEventRecord(i1, stream)); kinit.push_back({i0, i1}); }
     }
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
@@ -1573,7 +1577,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
         ms_kernel<T><<<dim3(mx, Gb), BLOCK, 0, stream>>>(a, d_m);
         launches++;
         st.ms_launches++;
-        st.ms_bytes += (uint64_t)Gb * nva * (B + 4);
+        st.ms_bytes += (uint64_t)Gb * nva * ((clean_ring ? 2 * B : B) + 4);  // + the visited words zeroed
       }
       if (o.timing) { CK(cudaEventRecord(m1, stream)); kms.push_back({m0, m1}); }
       if (clean_ring && !fused_clean) {  // the read slots back to zero (after late_fix read the skipped entries)
@@ -1684,15 +1688,20 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   for (auto &p : kcl) { float ms = 0; CK(cudaEventElapsedTime(&ms, p.first, p.second)); st.clean_ms += ms; }
   if (clean_ring && check_ring_enabled()) {
     CK(cudaMemsetAsync(flags, 0, 4, stream));
-    const size_t n16 = (size_t)R * G * gstride * B / 16;
+    const size_t n16 = (size_t)R * G * gstride * B / 16, v16 = (size_t)G * gstride * B / 16;
     ring_check_kernel<<<(uint32_t)std::min<size_t>((n16 + 255) / 256, 4096), 256, 0, stream>>>(
         reinterpret_cast<const uint4 *>(ring), n16, flags);
+    ring_check_kernel<<<(uint32_t)std::min<size_t>((v16 + 255) / 256, 4096), 256, 0, stream>>>(
+        reinterpret_cast<const uint4 *>(visited), v16, flags);
     uint32_t bad = 0;
     CK(cudaMemcpyAsync(&bad, flags, 4, cudaMemcpyDeviceToHost, stream));
     CK(cudaStreamSynchronize(stream));
-    if (bad) fail(IBFS_E_CUDA, "IBFS_CHECK_RING: a ring slot is not zero after the call");
+    if (bad) fail(IBFS_E_CUDA, "IBFS_CHECK_RING: a ring slot or visited word is not zero after the call");
   }
-  if (clean_ring) sc.mark_zero(ring_idx);  // every batch's clean-up is complete (harvest waited)
+  if (clean_ring) {  // every batch's clean-up is complete (harvest waited)
+    sc.mark_zero(ring_idx);
+    sc.mark_zero(vis_idx);
+  }
   st.depth_bytes += st.depth_rows_bytes;
   st.n_groups = n_groups;
   st.n_launches = launches;

@@ -401,7 +401,8 @@ __global__ void init_ctrl_kernel(BatchArgs<T> a, uint32_t first_dir) {
     }
 }
 
-// Zero the group's visited words and the snapshot slots of levels 0 and 1 (a2); when
+// Zero the group's visited words and the snapshot slots of levels 0 and 1 (a2; with the
+// clean ring they are zero already: ms_kernel / the clean-up passes left them so); when
 // level 1 runs bottom-up, enqueue every vertex of degree <= HUB_T (all are unvisited for
 // some active instance unless they are the source of every active instance -- the
 // expand skips those).
@@ -419,8 +420,8 @@ __global__ void __launch_bounds__(BLOCK) init_state_kernel(BatchArgs<T> a, uint3
   for (size_t v = (size_t)blockIdx.x * BLOCK + threadIdx.x; v < nvr; v += stride) {
     const bool in = v < a.nva;
     if (in) {
-      st(vis + v, z);
-      if (!a.clean_ring) {
+      if (!a.clean_ring) {  // clean ring: visited and the slots are zero already
+        st(vis + v, z);
         st(s0 + v, z);
         st(s1 + v, z);
       }
@@ -1371,6 +1372,94 @@ __device__ void commit_flush(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, in
   }
 }
 
+// Sparse commit with the clean ring: only the marked 32-vertex chunks can
+// hold bits of S_l (every write of the level marked its chunk and the slot started at
+// zero), so the warps of the whole grid scan the group's chunk map (16 flags per lane and
+// step) and commit each marked chunk warp-cooperatively, lane = vertex: mask S_l with
+// ~visited, visited |= S_l, the late-list entry, the top-down queue classes (no bottom-up
+// queue: the next level is top-down), the counters.  The frontier bitmap is not rewritten:
+// a sparse commit forces the next level top-down, only bottom-up levels read the bitmap,
+// and the next dense commit rewrites it whole.  Each taking part CTA flushes once.
+template <typename T>
+__device__ void commit_sparse_chunks(const BatchArgs<T> &a, CommitSmem<T> &cm, int g, int lc, uint32_t rank,
+                                     uint32_t K) {
+  constexpr int NP = WordBits<T>::value / 32;
+  const int lane = threadIdx.x & 31;
+  GroupCtrl<T> *c = a.ctrl + g;
+  uint32_t *qlen = c->qlen[lc & 1];
+  T *N = snap(a, g, lc);
+  T *vis = a.visited + (size_t)g * a.gstride;
+  uint8_t *dfl = a.dirty + (size_t)g * a.nchunk32;
+  unsigned long long nf = 0, mf = 0, newp = 0;
+  T nacc = wzero_value<T>();
+  const size_t nc = a.nchunk32;
+  const size_t gw = (size_t)rank * NWARP + (threadIdx.x >> 5), nw = (size_t)K * NWARP;
+  const bool al = (reinterpret_cast<uintptr_t>(dfl) & 15u) == 0;
+  for (size_t c0 = gw * 512; c0 < nc; c0 += nw * 512) {  // 512 flags per warp step
+    const size_t cl = c0 + (size_t)lane * 16;
+    uint32_t f[4] = {0u, 0u, 0u, 0u};
+    if (al && cl + 16 <= nc) {
+      const uint4 x = *reinterpret_cast<const uint4 *>(dfl + cl);
+      f[0] = x.x; f[1] = x.y; f[2] = x.z; f[3] = x.w;
+    } else {
+      for (int b = 0; b < 16; ++b)
+        if (cl + b < nc && dfl[cl + b]) f[b >> 2] |= 1u << (8 * (b & 3));
+    }
+    uint32_t hit = 0;  // bit b: flag b of this lane's 16 is set
+#pragma unroll
+    for (int b = 0; b < 16; ++b) hit |= ((f[b >> 2] >> (8 * (b & 3))) & 0xffu) ? (1u << b) : 0u;
+    uint32_t lanes = __ballot_sync(FULL, hit != 0);
+    while (lanes) {
+      const int src = __ffs(lanes) - 1;
+      lanes &= lanes - 1;
+      uint32_t h = __shfl_sync(FULL, hit, src);
+      while (h) {
+        const int b = __ffs(h) - 1;
+        h &= h - 1;
+        const size_t ch = c0 + (size_t)src * 16 + b;
+        const size_t v = ch * 32 + lane;
+        const bool in = v < a.nva;
+        T n = wzero_value<T>(), vv = wzero_value<T>();
+        uint32_t d = 0;
+        if (in) {
+          n = ld(N + v);
+          vv = ld(vis + v);
+          d = __ldg(a.deg + v);
+        }
+        const T m = wandn(n, vv);  // an unfiltered top-down OR may have set visited bits
+        if (in && !weq(m, n)) st(N + v, m);
+        const bool nz = !wzero(m);
+        if (nz) {
+          st(vis + v, wor(vv, m));
+          nf++;
+          mf += d;
+          newp += wpopc(m);
+          nacc = wor(nacc, m);
+        }
+        const uint32_t lb = __ballot_sync(FULL, nz);  // the late list (skipped level)
+        if (lb) {
+          const int leader = __ffs(lb) - 1;
+          uint32_t base0 = 0;
+          if (lane == leader) base0 = atomicAdd(a.late_n + g, (uint32_t)__popc(lb));
+          base0 = __shfl_sync(FULL, base0, leader);
+          const uint32_t i = base0 + __popc(lb & lanemask_lt());
+          if (nz && i < a.late_cap)
+            a.late[(size_t)g * a.late_cap + i] = ((unsigned long long)lc << 32) | (unsigned long long)v;
+        }
+        const bool qd = d > 0 && d <= (uint32_t)HUB_T, light = d <= (uint32_t)LIGHT_DEG;
+        queue_push(a, g, qlen, Q_TDL, nz && qd && light, (uint32_t)v);
+        queue_push(a, g, qlen, Q_TDH, nz && qd && !light, (uint32_t)v);
+        push_hub_chunks(a, g, qlen, Q_TDC, nz && d > (uint32_t)HUB_T, (uint32_t)v);
+        if (lane == 0) dfl[ch] = 0;  // consumed
+      }
+    }
+  }
+  float bc[NP];
+#pragma unroll
+  for (int p = 0; p < NP; ++p) bc[p] = 0.f;
+  commit_flush(a, cm, g, lc, 1u, K, nf, mf, newp, nacc, bc, true);
+}
+
 // Grid-wide barrier of a cooperative launch (every CTA resident): sense-reversing, one
 // counter and one generation word per batch.
 __device__ __forceinline__ void grid_barrier(uint32_t *bar) {
@@ -1435,19 +1524,25 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
 #pragma unroll
     for (int p = 0; p < NP; ++p) bc[p] = 0.f;
     for (int j = tid; j < WordBits<T>::value; j += BLOCK) cm.bcnt[j] = 0.f;
+    // each group's commit kind, from state fixed before this launch: read here, before
+    // this CTA arrives for any group (a group's last CTA rewrites dir / td_mark, which
+    // commit_sparse reads, once every CTA has arrived for it)
+    __shared__ uint8_t s_sparse[MAX_G];
+    for (int g = tid; g < a.G; g += BLOCK) s_sparse[g] = (!a.ctrl[g].done && commit_sparse(a, a.ctrl + g, lc)) ? 1 : 0;
     __syncthreads();
     for (size_t w = blockIdx.x; w < total; w += gridDim.x) {
       const int g = (int)(w / tpg);
       if (g != cur_g) {
         if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc, sparse);
         cur_g = g;
-        sparse = !a.ctrl[g].done && commit_sparse(a, a.ctrl + g, lc);
+        sparse = s_sparse[g] != 0;
         ntiles = 0;
         nf = mf = newp = 0;
         nacc = wzero_value<T>();
       }
       if (a.ctrl[g].done) continue;  // finished before this launch (stable)
       const uint32_t tix = (uint32_t)(w % tpg);
+      if (sparse && a.clean_ring) continue;  // the chunk scan below commits it
       if (tid == 0 && !sparse) {
         // the commit streams S_l, visited and the degrees of its tiles: ask the TMA unit to
         // prefetch this group's tile two tiles (of this CTA) ahead into L2
@@ -1459,6 +1554,14 @@ __global__ void __launch_bounds__(BLOCK, IBFS_EXPAND_MINB) level_kernel(BatchArg
       ++ntiles;
     }
     if (cur_g >= 0 && ntiles) commit_flush(a, cm, cur_g, lc, ntiles, tpg, nf, mf, newp, nacc, bc, sparse);
+    if (a.clean_ring) {
+      const uint32_t K = min(gridDim.x, max(1u, (uint32_t)((a.nchunk32 + NWARP * 2048 - 1) / (NWARP * 2048))));
+      for (int g = 0; g < a.G; ++g) {
+        if (!s_sparse[g]) continue;
+        const uint32_t rank = (blockIdx.x + gridDim.x - (uint32_t)(((size_t)g * K) % gridDim.x)) % gridDim.x;
+        if (rank < K) commit_sparse_chunks(a, cm, g, lc, rank, K);
+      }
+    }
     grid_barrier(a.gbar);
   }
   if (tid == 0 && blockIdx.x == 0) {
@@ -2120,8 +2223,11 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
   const size_t nvr = ((size_t)a.nva + 31) & ~(size_t)31;  // warp-uniform trip count
   for (size_t v = (size_t)blockIdx.x * BLOCK + tid; v < nvr; v += (size_t)gridDim.x * BLOCK) {
     const bool in = v < a.nva;
-    const T x = in ? ldg(vis + v) : wzero_value<T>();
+    // coherent load: with the clean ring this thread zeroes the word below (the
+    // non-coherent path could be ordered after that store)
+    const T x = in ? ld(vis + v) : wzero_value<T>();
     const uint32_t d = in ? __ldg(a.deg + v) : 0u;
+    if (a.clean_ring && in && !wzero(x)) st(const_cast<T *>(vis) + v, wzero_value<T>());  // visited back to zero
     const uint32_t any = __ballot_sync(FULL, !wzero(x) && d != 0);
     if (!any) continue;
     uint32_t m[NP];

@@ -4,7 +4,7 @@
 set -u
 OUT=gpurun_out/${1:-r02l}; mkdir -p "$OUT"
 python -c "import __graft_entry__ as e; e.build()" > "$OUT/build.log" 2>&1 || { cat "$OUT/build.log"; exit 1; }
-GOLDEN_THREADS=${GOLDEN_THREADS:-8} source tools/box_golden.sh
+[ -n "${GOLDEN_THREADS:-}" ] && source tools/box_golden.sh; GOLDEN_PID=${GOLDEN_PID:-}
 CFG=${CFG:-c5}
 timeout 900 python bench.py --config $CFG --no-e2e --no-cpu-baseline --json-out "$OUT/bench_$CFG.json" > "$OUT/bench_$CFG.log" 2>&1
 timeout 1500 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
@@ -18,6 +18,9 @@ for spec in ${SPECS:-"level_kernel:1:4 depth_tma_kernel:0:1"}; do
     -o "$OUT/full_${k}_$CFG" $B > "$OUT/full_${k}_$CFG.log" 2>&1
   echo "rc=$?" >> "$OUT/full_${k}_$CFG.log"
 done
+# c4 APSP as one call per step (all 2,048 groups): the per-call host return amortised
+timeout 900 python bench.py --config c4 --groups-per-rank 2048 --steps 3 --warmup 3 --no-e2e --no-cpu-baseline \
+  --json-out "$OUT/bench_c4_onecall.json" > "$OUT/bench_c4_onecall.log" 2>&1
 sleep ${GOLDEN_EXTRA:-0}
-kill $GOLDEN_PID 2>/dev/null
+[ -n "$GOLDEN_PID" ] && kill $GOLDEN_PID 2>/dev/null
 echo done > "$OUT/DONE"

@@ -24,6 +24,12 @@ FULL_METRICS = [
     ("l1tex__t_sector_hit_rate.pct", "L1hit%"),
     ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "SM%"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps%"),
+    ("smsp__thread_inst_executed_per_inst_executed.ratio", "lanes/inst"),
+    ("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "ld_sectors"),
+    ("l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum", "ld_requests"),
+    ("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "smem_wavefronts"),
+    ("l1tex__data_pipe_lsu_wavefronts_mem_shared.avg.pct_of_peak_sustained_elapsed", "smem%"),
+    ("smsp__inst_executed.sum", "warp_inst"),
     ("launch__registers_per_thread", "regs"),
     ("launch__grid_size", "grid"),
 ]
@@ -84,6 +90,13 @@ def full(reps):
                        f"{d.get('dram_wr', 0) / 1e6:.1f} | {gbs:.0f} | {d.get('dram%', 0):.1f} | {d.get('L2hit%', 0):.1f} | "
                        f"{d.get('L2thr%', 0):.1f} | {d.get('L1hit%', 0):.1f} | {d.get('SM%', 0):.1f} | "
                        f"{d.get('warps%', 0):.1f} | {d.get('regs', '')} | {d.get('grid', '')} |")
+    out += ["", "| report | kernel | lanes / inst | ld sectors / request | smem wavefronts (M) | smem % | warp inst (M) |",
+            "|---|---|---|---|---|---|---|"]
+    for rep in reps:
+        for d in raw(rep):
+            spr = d.get("ld_sectors", 0) / d["ld_requests"] if d.get("ld_requests") else 0
+            out.append(f"| {rep.split('/')[-1]} | `{d['kernel']}` | {d.get('lanes/inst', 0):.1f} | {spr:.2f} | "
+                       f"{d.get('smem_wavefronts', 0) / 1e6:.1f} | {d.get('smem%', 0):.1f} | {d.get('warp_inst', 0) / 1e6:.1f} |")
     return "\n".join(out)
 
 

@@ -12,7 +12,7 @@ timeout 1500 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byt
   python bench.py --config $CFG --steps 8 --warmup 3 --no-e2e --no-cpu-baseline > "$OUT/launches_$CFG.log" 2>&1
 echo "rc=$?" >> "$OUT/launches_$CFG.log"
 B="python bench.py --config $CFG --steps 1 --warmup 0 --no-e2e --no-cpu-baseline --no-clocks"
-for spec in ${SPECS:-"level_kernel:1:4 depth_tma_kernel:0:1"}; do
+for spec in ${SPECS:-level_kernel:1:4 depth_tma_kernel:0:1}; do
   IFS=: read k s c <<< "$spec"
   timeout 1200 ncu --set full --clock-control none --import-source on -k regex:$k -s $s -c $c \
     -o "$OUT/full_${k}_$CFG" $B > "$OUT/full_${k}_$CFG.log" 2>&1

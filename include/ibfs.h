@@ -256,7 +256,10 @@ typedef struct {
                    skipped levels excluded) + the late-list fix-ups; with the clean ring
                    at W = 128 the depth kernel also zeroes each loaded run (B per vertex,
                    group and loaded level, bulk stores) and clean_bytes excludes them;
-     ms_bytes      the m_s pass: (B + 4) per vertex and group (final words + degrees). */
+     ms_bytes      the m_s pass: (B + 4) per vertex and group (final words + degrees); with
+                   the clean ring also B per vertex and group (visited zeroed) and B per
+                   vertex, group and loaded level of the final flush (the ring slots it
+                   returns to zero; IBFS_MS_CLEAN=0 leaves them to ring_clean_kernel). */
   uint64_t commit_bytes_moved, depth_rows_bytes, ms_bytes;
   double ms_ms;                  /* m_s pass + late-list / isolated-source fix-ups (opts.timing) */
   uint64_t ms_launches;

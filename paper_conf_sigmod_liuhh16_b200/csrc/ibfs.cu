@@ -1122,6 +1122,11 @@ uint32_t bu_probe_mode() {
   return m;
 }
 
+bool env_flag(const char *name, bool dflt) {
+  const char *e = std::getenv(name);
+  return e ? e[0] == '1' : dflt;
+}
+
 // Clean ring unless IBFS_CLEAN_RING=0 (A/B runs: the commits clear the next
 // slot every level, as in round 1).  IBFS_CHECK_RING=1 (tests) verifies after every call
 // that the ring is all zero again and fails with IBFS_E_CUDA otherwise.
@@ -1140,6 +1145,10 @@ bool fused_clean_enabled() {
     const char *e = std::getenv("IBFS_FUSED_CLEAN");
     return e && e[0] == '1';
   }();
+  return on;
+}
+bool ms_clean_enabled() {
+  static const bool on = env_flag("IBFS_MS_CLEAN", true);
   return on;
 }
 bool check_ring_enabled() {
@@ -1397,6 +1406,10 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
   a.pol.max_depth = o.max_depth;
   a.pol.bu_probe = bu_probe_mode();
   a.pol.split_rel = split_rel_default();
+  {  // A/B: profiles/r02/td_scheck (1: c5 +2 %)
+    const char *e = std::getenv("IBFS_TD_SCHECK");
+    a.pol.td_scheck = (e && e[0] >= '0' && e[0] <= '2') ? (uint32_t)(e[0] - '0') : 1u;
+  }
   a.pol.sched_len = std::min<uint32_t>(o.schedule_len, MAXL);
   for (uint32_t i = 0; i < a.pol.sched_len; ++i) a.pol.sched[i] = (o.schedule[i] == 'B' || o.schedule[i] == 1) ? 1 : 0;
   uint32_t first_dir = 0;
@@ -1416,6 +1429,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
     uint32_t gb0 = 0, Gb = 0, rows = 0;
     int level = 0, slot = 0;
     int fused_from = 1 << 30;  // levels >= this were zeroed by the depth kernel (fused clean)
+    int ms_from = 1 << 30;     // levels >= this were zeroed by the m_s pass
     cudaEvent_t done = nullptr;
   } pend;
   // host side of a finished batch: per-source outputs, level records, byte models, times
@@ -1475,6 +1489,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
         if (clean_ring) {
           if (L.flags & 1u) st.clean_bytes += (uint64_t)L.nf * B;
           else if (l >= pb.fused_from) st.depth_bytes += (uint64_t)nva * B;  // the depth kernel's zero stores
+          else if (l >= pb.ms_from) st.ms_bytes += (uint64_t)nva * B;        // the m_s pass's zero stores
           else st.clean_bytes += (uint64_t)nva * B;
         }
         // depth kernel: a loaded level's snapshot is read once; a skipped level's new
@@ -1535,6 +1550,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
     // depth flush: rows from snapshots [l0, l1] (first flush writes every byte)
     int flushed = -1;  // levels <= flushed are already in the rows
     int fused_from = 1 << 30;
+    int ms_from = 1 << 30;
     bool batch_iso = false;  // a source of this batch is isolated (its own zero is a fix-up)
     for (uint32_t r = 0; r < rows_in_batch; ++r) {
       const uint32_t v = sources[(size_t)gb0 * W + r];
@@ -1548,6 +1564,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
       const int first = flushed < 0 ? 1 : 0;
       CUtensorMap tmap;
       bool fused_clean = false;  // the depth kernel zeroes the runs it loaded (clean ring, W = 128)
+      bool clean_in_ms = false;  // the m_s pass zeroed them
       if (first && depth_tma_enabled() && make_rows_tensor_map(&tmap, a.out, nv, rows_in_batch, W)) {
         fused_clean = clean_ring && B == 16 && fused_clean_enabled();
         if (fused_clean) fused_from = std::min(fused_from, flushed + 1);
@@ -1574,13 +1591,20 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
       if (final_flush) {  // m_s from the final visited words (reading #11)
         const uint32_t mx = (uint32_t)std::max<uint64_t>(
             1, std::min<uint64_t>(((uint64_t)nva + BLOCK - 1) / BLOCK, std::max<uint64_t>(1, (uint64_t)g->num_sms * 4 / Gb)));
-        ms_kernel<T><<<dim3(mx, Gb), BLOCK, 0, stream>>>(a, d_m);
+        // clean ring: the m_s pass also zeroes this flush's loaded slots (IBFS_MS_CLEAN=0:
+        // the separate ring_clean_kernel pass)
+        const bool ms_clean = clean_ring && !fused_clean && ms_clean_enabled();
+        ms_kernel<T><<<dim3(mx, Gb), BLOCK, 0, stream>>>(a, d_m, ms_clean ? flushed + 1 : 1, ms_clean ? l1 : 0);
+        if (ms_clean) {
+          clean_in_ms = true;
+          ms_from = std::min(ms_from, flushed + 1);
+        }
         launches++;
         st.ms_launches++;
         st.ms_bytes += (uint64_t)Gb * nva * ((clean_ring ? 2 * B : B) + 4);  // + the visited words zeroed
       }
       if (o.timing) { CK(cudaEventRecord(m1, stream)); kms.push_back({m0, m1}); }
-      if (clean_ring && !fused_clean) {  // the read slots back to zero (after late_fix read the skipped entries)
+      if (clean_ring && !fused_clean && !clean_in_ms) {  // the read slots back to zero (after late_fix read the skipped entries)
         cudaEvent_t c0 = nullptr, c1 = nullptr;
         if (o.timing) { c0 = timer.next(); c1 = timer.next(); CK(cudaEventRecord(c0, stream)); }
         const uint32_t cx = (uint32_t)std::max<uint64_t>(
@@ -1668,6 +1692,7 @@ void run_typed(const ibfs_graph *g, const uint32_t *sources, uint32_t n,
     cur.rows = rows_in_batch;
     cur.level = level;
     cur.fused_from = fused_from;
+    cur.ms_from = ms_from;
     cur.slot = batch_no & 1;
     cur.done = timer.next();  // not from `chk`: its events are recycled every batch
     CK(cudaEventRecord(cur.done, stream));

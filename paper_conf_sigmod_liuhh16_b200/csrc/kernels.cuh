@@ -135,6 +135,7 @@ struct Policy {
   uint32_t max_depth;  // k-hop cap (0 = unbounded)
   uint32_t bu_probe;   // frontier-bitmap probes in BU: 0 never, 1 sparse frontiers (default), 2 always
   float split_rel;     // > 0: also top-down when m_f(j) * split_rel < max over active j' of m_f(j')
+  uint32_t td_scheck;  // top-down ORs read S_l[w] first: 1 unfiltered ones, 2 all (A/B knob IBFS_TD_SCHECK)
   uint8_t sched[MAXL];  // 0 TD / 1 BU for level l at index l-1
 };
 
@@ -608,7 +609,11 @@ __device__ void item_td(const BatchArgs<T> &a, ExpandSmem &sm, TileQueue<T> &tq,
       if (w[u] != 0xffffffffu) {
         insp++;
         gath += filt ? 1u : 0u;
-        const T b = filt ? wandn(fw[u], ldg(vis + w[u])) : fw[u];
+        T b = filt ? wandn(fw[u], ldg(vis + w[u])) : fw[u];
+        // IBFS_TD_SCHECK: skip the RED.OR when S_l[w] already holds the bits (an L2 read
+        // instead of a read-modify-write; a stale read shows a subset of the bits, so a
+        // needed OR is never skipped)
+        if (a.pol.td_scheck > (filt ? 1u : 0u) && !wzero(b)) b = wandn(b, ldcg_w(N + w[u]));
         if (!wzero(b)) {
           red_or(N + w[u], b);
           writes++;
@@ -796,7 +801,8 @@ __device__ void hub_td(const BatchArgs<T> &a, ExpandSmem &sm, int g, const HubCh
       if (w[u] != 0xffffffffu) {
         insp++;
         gath += filt ? 1u : 0u;
-        const T b = filt ? wandn(f, ldg(vis + w[u])) : f;
+        T b = filt ? wandn(f, ldg(vis + w[u])) : f;
+        if (a.pol.td_scheck > (filt ? 1u : 0u) && !wzero(b)) b = wandn(b, ldcg_w(N + w[u]));
         if (!wzero(b)) {
           red_or(N + w[u], b);
           writes++;
@@ -2199,10 +2205,12 @@ __global__ void __launch_bounds__(DTHREADS + 32, IBFS_DTMA_MINB)
 // M of the warp's vertices reached by instance 32p + i, and the degree-weighted count is
 // sum_b popc(M & D_b) << b over the degree bit planes D_b = ballot(bit b of deg).
 template <typename T>
-__global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long long *m_out) {
+__global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long long *m_out, int zl0, int zl1) {
   constexpr int W = WordBits<T>::value;
   constexpr int NP = W / 32;
   __shared__ unsigned long long s_m[W];
+  __shared__ T *s_zero[DMAXL];  // clean ring: the loaded snapshot slots this pass zeroes
+  __shared__ int s_nz;
   const int g = blockIdx.y;
   const int rows = group_rows(a, g);
   // a group finished at init (every source isolated) never zeroed its visited words; its
@@ -2210,7 +2218,19 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
   if (rows == 0 || a.ctrl[g].last_level == 0xffffffffu) return;
   const int tid = threadIdx.x, lane = tid & 31;
   for (int j = tid; j < W; j += BLOCK) s_m[j] = 0;
+  if (tid == 0) {
+    // zl0 <= zl1: also return the loaded slots of levels [zl0, zl1] to zero (the clean
+    // ring's pass fused into this ALU-bound one: the stores overlap the bit transposes)
+    const GroupCtrl<T> *c = a.ctrl + g;
+    const int last = min((int)c->last_level, min(zl1, 127));
+    const unsigned long long sk0 = c->skip_lv[0], sk1 = c->skip_lv[1];
+    int n = 0;
+    for (int l = zl0; l <= last && n < DMAXL; ++l)
+      if (((l < 64 ? sk0 >> l : sk1 >> (l - 64)) & 1ull) == 0) s_zero[n++] = snap(a, g, l);
+    s_nz = n;
+  }
   __syncthreads();
+  const int nzs = s_nz;
   const T *vis = a.visited + (size_t)g * a.gstride;
   unsigned long long acc[NP];
   uint32_t cnt[NP][8];  // popcounts per (piece, degree bit plane < 8), weighted at the end
@@ -2228,6 +2248,8 @@ __global__ void __launch_bounds__(BLOCK) ms_kernel(BatchArgs<T> a, unsigned long
     const T x = in ? ld(vis + v) : wzero_value<T>();
     const uint32_t d = in ? __ldg(a.deg + v) : 0u;
     if (a.clean_ring && in && !wzero(x)) st(const_cast<T *>(vis) + v, wzero_value<T>());  // visited back to zero
+    if (in)
+      for (int z = 0; z < nzs; ++z) st_cs(s_zero[z] + v, wzero_value<T>());
     const uint32_t any = __ballot_sync(FULL, !wzero(x) && d != 0);
     if (!any) continue;
     uint32_t m[NP];

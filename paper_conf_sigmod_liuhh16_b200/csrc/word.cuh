@@ -134,6 +134,12 @@ __device__ __forceinline__ void st(unsigned long long *p, unsigned long long v) 
 __device__ __forceinline__ void st(u128 *p, u128 v) {
   *reinterpret_cast<ulonglong2 *>(p) = make_ulonglong2(v.lo, v.hi);
 }
+// streaming (evict-first) stores: words no kernel of this batch reads again
+__device__ __forceinline__ void st_cs(uint32_t *p, uint32_t v) { __stcs(p, v); }
+__device__ __forceinline__ void st_cs(unsigned long long *p, unsigned long long v) { __stcs(p, v); }
+__device__ __forceinline__ void st_cs(u128 *p, u128 v) {
+  __stcs(reinterpret_cast<ulonglong2 *>(p), make_ulonglong2(v.lo, v.hi));
+}
 
 // Atomic OR without return (compiles to RED.OR).  No 128-bit atomicOr exists, so W = 128
 // issues two independent 64-bit reductions; OR is bitwise, so the halves commute

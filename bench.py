@@ -200,9 +200,9 @@ def make_roofline(config, sts, step_ms):
           "algorithmic_bytes_per_launch": (b / live if live else None),
           "launches": nl, "launches_live": live,
           "model": "DESIGN.md §5 = SURVEY.md §8(d): expand 8+B per frontier, 4+B per inspection, B per write; "
-                   "commit 2B per vertex (dense scan; the clean ring clears each read slot once, in the clean "
-                   "kernel: B per vertex and loaded level) + B per new vertex; depth rows i*|V| + B per "
-                   "loaded snapshot",
+                   "commit 2B per vertex (dense scan; the clean ring clears each read slot once, in the m_s "
+                   "pass or the clean kernel: B per vertex and loaded level) + B per new vertex; depth rows "
+                   "i*|V| + B per loaded snapshot",
           "share_of_step": round(ms / step_ms, 4) if step_ms else None,
           "all_kernels": {k: {"GB/s": gbs(v[0], v[1]), "ms": round(v[1], 3), "launches": v[3], "live": v[2],
                               "bytes_per_live_launch": (v[0] / v[2] if v[2] else None)} for k, v in kern.items()},

@@ -48,7 +48,7 @@ def parse(argv=None):
     ap.add_argument("--groups-in-flight", type=int, default=0, help="groups per launch batch (0 = library auto)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--direction", default="auto")
-    ap.add_argument("--alpha", type=float, default=4.0)
+    ap.add_argument("--alpha", type=float, default=3.0)
     ap.add_argument("--beta", type=float, default=24.0)
     ap.add_argument("--split-div", type=float, default=512.0)
     ap.add_argument("--group-bits", type=int, default=0, help="instances per group (0 = the config's, 128)")

@@ -160,7 +160,7 @@ typedef struct {
   uint32_t bu_from;           /* for IBFS_DIR_BU_FROM (level >= 1) */
   const uint8_t *schedule;    /* host array of 'T'/'B' for IBFS_DIR_SCHEDULE */
   uint32_t schedule_len;
-  float alpha;                /* TD->BU when m_f * alpha > m_u (default 4.0) */
+  float alpha;                /* TD->BU when m_f * alpha > m_u (default 3.0) */
   float beta;                 /* BU->TD when n_f * beta < nv_active (default 24.0) */
   uint32_t groups_in_flight;  /* groups per launch batch; 0 = auto from nv and memory */
   void *cuda_stream;          /* cudaStream_t to launch on; NULL = legacy default stream.

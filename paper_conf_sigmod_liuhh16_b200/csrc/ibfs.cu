@@ -1084,7 +1084,7 @@ extern "C" void ibfs_run_opts_default(ibfs_run_opts *o) {
   std::memset(o, 0, sizeof(*o));
   o->direction = IBFS_DIR_AUTO;
   o->bu_from = 2;
-  o->alpha = 4.0f;
+  o->alpha = 3.0f;  // profiles/r02/direction: c3 +4 %, c4 +3 %, c5 +0.5 % over 4
   o->beta = 24.0f;
   o->split = IBFS_SPLIT_AUTO;
   o->split_mod = 2;

@@ -219,7 +219,7 @@ class Graph:
 
     # ---- traversal -----------------------------------------------------------------
     def run(self, sources, group_bits: int = 128, out="device", direction: str = "auto",
-            schedule: str | None = None, bu_from: int = 2, alpha: float = 4.0, beta: float = 24.0,
+            schedule: str | None = None, bu_from: int = 2, alpha: float = 3.0, beta: float = 24.0,
             groups_in_flight: int = 0, stream=None, timing: bool = False, want_m: bool = True,
             want_digest: bool = False, level_cap: int = 130, split: str = "auto",
             split_mod: int = 2, split_div: float = 512.0, max_depth: int | None = None,
